@@ -1,0 +1,233 @@
+/*
+ * sassi.h — C ABI of the B200-native SASSI instrumentation-handler analysis path.
+ *
+ * What this library computes (PAPER.md = /root/reference/PAPER.md, "Lnnn" = its line):
+ *   Stephenson et al., "Flexible Software Profiling of GPU Architectures" (SASSI), ISCA'15.
+ *   SASSI calls a user handler at every instrumented SASS instruction (L181-L187, §3.1-3.2).
+ *   The paper's four case-study handlers are folded here over warp-wide instruction records:
+ *     - SASSI_H_BRANCH    conditional-branch divergence   (§5, Fig.4)
+ *     - SASSI_H_MEMDIV    memory address divergence       (§6, Fig.6)
+ *                         in 32 B sectors (the paper's "line", L367) and 128 B lines
+ *     - SASSI_H_VALUE     value profiling: constant bits + scalar writes (§7, Fig.9)
+ *     - SASSI_H_INSTCOUNT per-thread dynamic-instruction counts for error-injection
+ *                         site selection (§8.1)
+ *   The handler semantics (which lanes count, init values, counter widths) are spelled out in
+ *   DESIGN.md §3 ("Readings"); every table entry is an integer fold, so results are exact.
+ *
+ * ---------------------------------------------------------------------------------------------
+ * RECORD FORMAT "SRF1" (all little-endian, all buffers DEVICE memory unless stated otherwise)
+ * ---------------------------------------------------------------------------------------------
+ *  The static "where/what" of SASSI (L181-L187) is a site table registered once per context:
+ *    sassi_site { pc, flags, mem_width, domain, n_gpr_dst, reg_num[4] }          (16 B)
+ *  mirroring the static parts of SASSIBeforeParams.insEncoding / SASSIMemoryParams.properties,
+ *  width, domain (Fig.2b/c, L157-L173) and SASSIRegisterParams.GetNumGPRDsts/GetRegNum (L555).
+ *
+ *  The dynamic part is one 16 B header per dynamic warp-instruction ("record"):
+ *    sassi_hdr { pc, warp, active, mask2 }
+ *      pc     instruction address (SASSIBeforeParams.GetInsAddr, L159)
+ *      warp   global warp id; thread id = 32*warp + lane (L629 "thread ID")
+ *      active lanes executing the instruction (__ballot(1), L239 l.13)
+ *      mask2  COND_BRANCH sites: lanes whose direction is "taken" (GetDirection, L237 l.8)
+ *             all other sites: guard-predicate-true lanes (instrWillExecute, L173, L363 l.4)
+ *  plus payload rows, each a full warp wide, in record order:
+ *    addr row  uint64_t[32]  one per record at a site with SASSI_F_MEM (any domain):
+ *              lane l's effective address (SASSIMemoryParams.GetAddress, L165)
+ *    val rows  uint32_t[32]  n_gpr_dst rows per record at a site with n_gpr_dst > 0:
+ *              lane l's value written to destination d (GetRegValue, L555)
+ *  Rows exist for every record whose pc is registered, whatever its masks (even active == 0).
+ *  Records whose pc is NOT registered carry no rows. Lanes outside the relevant mask may hold
+ *  any value. Row content outside the masks is never read by the fold.
+ *
+ *  chunk_base[ceil(n/SASSI_CHUNK)+1]: for chunk c, the index of the first addr row and first
+ *  val row belonging to a record with index >= c*SASSI_CHUNK; entry [n_chunks] holds the
+ *  totals. It is an index over the row streams so independent workers can start mid-stream;
+ *  sassi_index_records() builds it on the device from the headers when the producer did not.
+ *
+ * ---------------------------------------------------------------------------------------------
+ * TABLE IMAGE (what sassi_read_tables returns): one flat uint64_t array, offsets from
+ * sassi_table_layout(n_sites, n_warps). S = n_sites in REGISTRATION order, W = n_warps.
+ * ---------------------------------------------------------------------------------------------
+ *   diag[8]        n_records, n_invalid (active==0), n_unknown_pc, n_bad_warp (instcount record
+ *                  with warp >= W), n_sites, n_warps, handler_mask, SASSI_ABI_VERSION
+ *   br[S][5]       totalBranches, activeThreads, takenThreads, takenNotThreads,
+ *                  divergentBranches                              (BranchStats, Fig.4 l.27-33)
+ *   mem[S][4]      warp accesses, active lanes, distinct 32 B sectors, distinct 128 B lines
+ *   val[S][2]      warp executions, thread executions ("weight", Fig.9)
+ *   ones[S][4]     constantOnes[d]  (low 32 bits used; init 0xFFFFFFFF)   (Fig.9)
+ *   zeros[S][4]    constantZeros[d] (low 32 bits used; init 0xFFFFFFFF)   (Fig.9)
+ *   nonscalar[S][4] warp executions whose lanes did not all write the same value to dst d;
+ *                  the paper's isScalar[d] == (nonscalar[d] == 0)       (Fig.9)
+ *   h32[32][32]    sassi_counters[numActive-1][unique-1], unique = distinct 32 B sectors (Fig.6 l.33)
+ *   h128[32][32]   the same matrix with 128 B lines
+ *   counts[32*W]   per-thread eligible dynamic-instruction counts (§8.1 (4), L627)
+ *
+ * ---------------------------------------------------------------------------------------------
+ * CONVENTIONS
+ *   - Every function returns a sassi_status (0 = OK, < 0 = error); no exception crosses the ABI.
+ *   - Asynchronous CUDA faults surface as SASSI_ECUDA at the next call that synchronises.
+ *   - A context is bound to one device and is NOT thread-safe.
+ *   - The context owns its device tables and site hash; the caller owns record buffers and
+ *     streams. Record buffers must stay valid until the stream work of the call completes.
+ *   - `stream` arguments are cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - There is no CPU fallback: without a usable CUDA device every call fails (SASSI_ECUDA).
+ */
+#ifndef SASSI_H_
+#define SASSI_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SASSI_ABI_VERSION 1u
+#define SASSI_WARP_SIZE 32u
+#define SASSI_CHUNK 256u           /* records per chunk_base entry */
+#define SASSI_MAX_SITES 4096u      /* registered sites per context */
+#define SASSI_MAX_DST 4u           /* GPR destinations per instruction (e.g. 128-bit loads) */
+
+typedef enum sassi_status {
+  SASSI_OK = 0,
+  SASSI_EINVAL = -1,     /* bad argument (null pointer, bad flags, duplicate pc, ...)        */
+  SASSI_ECUDA = -2,      /* CUDA runtime error (message via sassi_strerror / last error)     */
+  SASSI_ENCCL = -3,      /* NCCL error or NCCL library not loadable                          */
+  SASSI_ENOSPC = -4,     /* too many sites / handler state does not fit shared memory         */
+  SASSI_ESTATE = -5,     /* call not valid in the context's current state                    */
+  SASSI_EMISMATCH = -6,  /* site tables differ across ranks in sassi_merge                   */
+  SASSI_EFORMAT = -7     /* record stream inconsistent with its row counts / chunk index     */
+} sassi_status;
+
+/* Handler kinds for sassi_attach_handler (bit mask). */
+enum {
+  SASSI_H_BRANCH = 1u,
+  SASSI_H_MEMDIV = 2u,
+  SASSI_H_VALUE = 4u,
+  SASSI_H_INSTCOUNT = 8u,
+  SASSI_H_ALL = 15u
+};
+
+/* sassi_site.flags — static instruction properties (insEncoding / properties). */
+enum {
+  SASSI_F_COND_BRANCH = 1u << 0, /* IsCondControlXfer (L159): mask2 = taken lanes              */
+  SASSI_F_CTRL = 1u << 1,        /* IsControlXfer                                            */
+  SASSI_F_MEM = 1u << 2,         /* IsMem: record carries an addr row                        */
+  SASSI_F_MEM_READ = 1u << 3,    /* IsMemRead / IsLoad                                       */
+  SASSI_F_MEM_WRITE = 1u << 4,   /* IsMemWrite / IsStore                                     */
+  SASSI_F_ATOMIC = 1u << 5,      /* IsAtomic                                                 */
+  SASSI_F_SYNC = 1u << 6,        /* IsSync                                                   */
+  SASSI_F_NUMERIC = 1u << 7,     /* IsNumeric                                                */
+  SASSI_F_TEXTURE = 1u << 8,     /* IsTexture                                                */
+  SASSI_F_WRITES_PRED = 1u << 9, /* writes a predicate register (error model, L621)          */
+  SASSI_F_WRITES_CC = 1u << 10,  /* writes the condition code (error model, L621)            */
+  SASSI_F_ALL = (1u << 11) - 1u
+};
+
+/* sassi_site.domain — SASSIMemoryParams.GetDomain (L167); memdiv counts GLOBAL only (L363 l.7). */
+enum { SASSI_D_GLOBAL = 0, SASSI_D_SHARED = 1, SASSI_D_LOCAL = 2, SASSI_D_CONST = 3, SASSI_D_TEX = 4 };
+
+typedef struct sassi_site {
+  uint32_t pc;         /* instruction address; must be unique; 0xFFFFFFFF is reserved          */
+  uint16_t flags;      /* SASSI_F_*; COND_BRANCH excludes MEM and n_gpr_dst > 0                 */
+  uint8_t mem_width;   /* bytes per lane access (GetWidth, L167); informational                 */
+  uint8_t domain;      /* SASSI_D_* (meaningful with SASSI_F_MEM)                               */
+  uint8_t n_gpr_dst;   /* 0..SASSI_MAX_DST GPR destinations (GetNumGPRDsts, L555)               */
+  uint8_t reg_num[4];  /* destination register numbers (GetRegNum, L555), for reports          */
+  uint8_t reserved[3];
+} sassi_site;          /* 16 B */
+
+typedef struct sassi_hdr {
+  uint32_t pc, warp, active, mask2;
+} sassi_hdr;           /* 16 B */
+
+typedef struct sassi_chunk_base {
+  uint64_t addr_row, val_row;
+} sassi_chunk_base;    /* 16 B */
+
+typedef struct sassi_records {
+  const sassi_hdr* hdr;                /* [n]                                                */
+  const uint64_t* addr;                /* [n_addr_rows][32] (may be NULL if n_addr_rows == 0) */
+  const uint32_t* val;                 /* [n_val_rows][32]  (may be NULL if n_val_rows == 0)  */
+  const sassi_chunk_base* chunk_base;  /* [ceil(n/SASSI_CHUNK)+1]                             */
+  uint64_t n_addr_rows, n_val_rows;
+} sassi_records;
+
+/* One error-injection site tuple (L629): kernel, dynamic invocation, thread, dynamic instruction
+ * index of that thread, seed to choose the destination register, seed to choose the bit. */
+typedef struct sassi_inj_site {
+  uint32_t kernel, invocation, thread, reg_seed, bit_seed, reserved;
+  uint64_t dyn_index;
+} sassi_inj_site;      /* 32 B */
+
+typedef struct sassi_layout {
+  uint64_t diag, br, mem, val, ones, zeros, nonscalar, h32, h128, counts, total; /* in u64 words */
+} sassi_layout;
+
+/* Offsets of the table image (host-only arithmetic; no device needed). */
+int sassi_table_layout(uint32_t n_sites, uint32_t n_warps, sassi_layout* out);
+
+/* Create a context on `device` for a program with the given static sites (HOST array, copied)
+ * and n_warps trace warps (per-thread counts cover 32*n_warps threads). The site hash (open
+ * addressing keyed by pc, L239 l.21-23 "find") is built here and uploaded.
+ * Errors: EINVAL (null/invalid site, duplicate pc), ENOSPC (n_sites > SASSI_MAX_SITES), ECUDA. */
+int sassi_ctx_create(struct sassi_ctx** out, int device, const sassi_site* sites, uint32_t n_sites,
+                     uint32_t n_warps);
+void sassi_ctx_destroy(struct sassi_ctx* ctx);
+
+/* Select which handlers run (SASSI_H_* mask) — the paper's "what" (L181-L187). Allowed only
+ * before the first consume or right after sassi_reset. Errors: EINVAL, ESTATE, ENOSPC. */
+int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
+
+/* Fold n records (DEVICE buffers) into the context's tables; asynchronous, stream-ordered.
+ * Tables accumulate across calls until sassi_reset. Errors: EINVAL, ESTATE (no handler), ECUDA. */
+int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, void* stream);
+
+/* Same fold from HOST buffers (pinned or pageable): the library copies slices to the device
+ * (double-buffered on `stream` plus an internal copy stream), consumes them, and returns after
+ * the stream work completes. recs->chunk_base is required (host). */
+int sassi_consume_host(struct sassi_ctx* ctx, const sassi_records* host_recs, uint64_t n,
+                       void* stream);
+
+/* Build chunk_base (DEVICE, ceil(n/SASSI_CHUNK)+1 entries) from device headers using the
+ * context's site table (row counts per record follow from the site of its pc). */
+int sassi_index_records(struct sassi_ctx* ctx, const sassi_hdr* hdr, uint64_t n,
+                        sassi_chunk_base* chunk_base_out, void* stream);
+
+/* Re-initialise all tables (CUPTI kernel-launch callback analogue, L217). Asynchronous. */
+int sassi_reset(struct sassi_ctx* ctx, void* stream);
+
+/* Copy the table image (sassi_table_layout(...).total words) to HOST memory; synchronises
+ * `stream` (CUPTI kernel-exit callback analogue, L217). Errors: EINVAL (n_words too small). */
+int sassi_read_tables(struct sassi_ctx* ctx, uint64_t* host_out, uint64_t n_words, void* stream);
+
+/* Device pointer to the live table image (owned by the context; read-only for the caller). */
+int sassi_tables_device(struct sassi_ctx* ctx, const uint64_t** dev_ptr, uint64_t* n_words);
+
+/* Exclusive scan of the per-thread counts and k draws of injection sites (L629), uniform over
+ * all eligible dynamic thread-instructions, with replacement, draw j from splitmix64(seed + j).
+ * out is a HOST array of k tuples; synchronises `stream`. Errors: ESTATE if the total is 0. */
+int sassi_sample_sites(struct sassi_ctx* ctx, uint32_t k, uint64_t seed, sassi_inj_site* host_out,
+                       void* stream);
+
+/* Multi-GPU: merge the tables of all ranks of `nccl_comm` (ncclComm_t) in place with one
+ * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits).
+ * Collective: every rank must call it. Errors: ENCCL, EMISMATCH (site tables differ). */
+int sassi_merge(struct sassi_ctx* ctx, void* nccl_comm, void* stream);
+
+/* NCCL bootstrap helpers (NCCL is loaded lazily with dlopen; only sassi_merge needs it). */
+int sassi_nccl_get_unique_id(void* out_128_bytes);
+int sassi_nccl_comm_create(void** comm_out, int nranks, int rank, const void* unique_id_128_bytes,
+                           int device);
+int sassi_nccl_comm_destroy(void* comm);
+
+/* Number of kernels this context launched so far (for the bench's launch count). */
+int sassi_kernel_launches(struct sassi_ctx* ctx, uint64_t* out);
+
+const char* sassi_strerror(int status);
+/* Message of the most recent failing call in this process (thread-local). */
+const char* sassi_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SASSI_H_ */
