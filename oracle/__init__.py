@@ -118,16 +118,20 @@ def table_init(n_sites: int, n_warps: int, handler_mask: int) -> np.ndarray:
 
 
 def consume(table: np.ndarray, sites: np.ndarray, n_warps: int, handler_mask: int,
-            hdr: np.ndarray, addr: np.ndarray | None, val: np.ndarray | None) -> np.ndarray:
-    """Fold records into ``table`` in place (and return it). addr: [rows,32] u64; val: [rows,32] u32."""
+            hdr: np.ndarray, addr: np.ndarray | None, val: np.ndarray | None,
+            n_addr_rows: int | None = None, n_val_rows: int | None = None) -> np.ndarray:
+    """Fold records into ``table`` in place (and return it). addr: [rows,32] u64; val: [rows,32] u32.
+    A row array may be None when no attached handler reads it; pass its row count instead."""
     sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
     hdr = np.ascontiguousarray(hdr, dtype=HDR_DTYPE)
-    addr = np.zeros((0, 32), np.uint64) if addr is None else np.ascontiguousarray(addr, np.uint64)
-    val = np.zeros((0, 32), np.uint32) if val is None else np.ascontiguousarray(val, np.uint32)
+    na = (0 if addr is None else np.asarray(addr).reshape(-1, 32).shape[0]) if n_addr_rows is None else n_addr_rows
+    nv = (0 if val is None else np.asarray(val).reshape(-1, 32).shape[0]) if n_val_rows is None else n_val_rows
+    addr = None if addr is None else np.ascontiguousarray(addr, np.uint64)
+    val = None if val is None else np.ascontiguousarray(val, np.uint32)
     assert table.dtype == np.uint64 and table.flags.c_contiguous
     rc = lib().oracle_consume(sites.ctypes.data, len(sites), n_warps, handler_mask,
-                              _ptr(hdr), len(hdr), _ptr(addr), addr.reshape(-1, 32).shape[0],
-                              _ptr(val), val.reshape(-1, 32).shape[0], table.ctypes.data)
+                              _ptr(hdr), len(hdr), _ptr(addr), na, _ptr(val), nv,
+                              table.ctypes.data)
     if rc != 0:
         raise ValueError("oracle_consume: record stream inconsistent with its rows (rc=%d)" % rc)
     return table

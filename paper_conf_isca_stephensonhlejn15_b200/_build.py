@@ -47,9 +47,16 @@ def build(force: bool = False, verbose: bool = False) -> dict:
         [os.path.join(INCLUDE, "sassi.h")]
     tgt = os.path.join(LIB, "libsassi.so")
     if srcs and (force or _stale(tgt, deps)):
+        from concurrent.futures import ThreadPoolExecutor
+        objdir = os.path.join(ROOT, "build", "obj")
+        os.makedirs(objdir, exist_ok=True)
+        objs = [os.path.join(objdir, os.path.basename(s) + ".o") for s in srcs]
+        with ThreadPoolExecutor(max_workers=min(8, len(srcs))) as ex:
+            list(ex.map(lambda so: _run([NVCC] + NVFLAGS + ["-I", INCLUDE, "-I", CSRC, "-c", "-o",
+                                                              so[1], so[0]], verbose),
+                        zip(srcs, objs)))
         tmp = tgt + ".tmp%d" % os.getpid()
-        _run([NVCC] + NVFLAGS + ["-I", INCLUDE, "-I", CSRC, "-shared", "-o", tmp] + srcs +
-             ["-ldl", "-lpthread"], verbose)
+        _run([NVCC] + ARCH + ["-shared", "-o", tmp] + objs + ["-ldl", "-lpthread"], verbose)
         os.replace(tmp, tgt)
     out["libsassi"] = tgt
     # device generator

@@ -1,0 +1,121 @@
+// common.cuh — internals shared by the libsassi.so translation units (never by the oracle).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "sassi.h"
+
+namespace sassi {
+
+constexpr uint32_t FULL = 0xFFFFFFFFu;
+constexpr uint32_t EMPTY_KEY = 0xFFFFFFFFu;
+constexpr int kConsumeThreads = 256;          // 8 warps per CTA
+constexpr int kWarpsPerCta = kConsumeThreads / 32;
+constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 30;  // keeps every smem u32 partial < 2^32
+
+// Packed per-site info word in the hash (bit layout).
+constexpr uint32_t I_SITE_MASK = 0xFFFu;      // site index (registration order), < 4096
+constexpr uint32_t I_BRANCH = 1u << 12;       // COND_BRANCH site
+constexpr uint32_t I_ADDR_ROW = 1u << 13;     // record carries an addr row (MEM, any domain)
+constexpr uint32_t I_MEMDIV = 1u << 14;       // MEM && GLOBAL: folded by the memdiv handler
+constexpr uint32_t I_NDST_SHIFT = 15;         // 3 bits: n_gpr_dst
+constexpr uint32_t I_ELIGIBLE = 1u << 18;     // instcount-eligible (R12)
+
+__host__ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
+  h ^= h >> 16;
+  h *= 0x85EBCA6Bu;
+  h ^= h >> 13;
+  h *= 0xC2B2AE35u;
+  h ^= h >> 16;
+  return h;
+}
+
+// Table image offsets (u64 words), same formulas as sassi_table_layout().
+struct Offsets {
+  uint64_t br, mem, val, ones, zeros, nonscalar, h32, h128, counts, total;
+};
+
+// Kernel parameter block of the fused consume kernel.
+struct ConsumeParams {
+  const uint4* hdr;                 // [n] headers (16 B each)
+  const uint64_t* addr;             // addr rows; row r at addr + 32 * (r - arow_base)
+  const uint32_t* val;              // val rows;  row r at val + 32 * (r - vrow_base)
+  const ulonglong2* cb;             // chunk index for the records of this launch
+  uint64_t n;                       // records in this launch (hdr[0] starts a chunk)
+  uint64_t arow_base, vrow_base;    // row index of addr[0] / val[0]
+  uint64_t arow_end, vrow_end;      // one past the last valid row index (bounds check)
+  const uint32_t* hash;             // [3][cap]: keys, info, cidx
+  uint32_t cap;                     // power of two
+  uint32_t nb, nm, nvw;             // smem counters: branch sites, memdiv sites, value words
+  uint32_t n_warps;                 // per-thread count coverage (32 * n_warps threads)
+  uint32_t nv;                      // value sites (flush map entries)
+  const uint32_t* flush_b;          // [nb] site index of branch compact slot
+  const uint32_t* flush_m;          // [nm] site index of memdiv compact slot
+  const uint32_t* flush_v;          // [nv][3] site index, word offset, n_dst
+  uint64_t* table;                  // device table image
+  Offsets off;
+  uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
+};
+
+}  // namespace sassi
+
+struct sassi_ctx {
+  int device = 0;
+  uint32_t S = 0, W = 0;
+  uint32_t mask = 0;
+  bool consumed = false;
+  std::vector<sassi_site> sites;
+  sassi::Offsets off{};
+  uint64_t checksum = 0;
+  // device state
+  uint64_t* d_table = nullptr;
+  uint32_t* d_hash = nullptr;       // [3][cap]
+  uint32_t cap = 0;
+  uint32_t nb = 0, nm = 0, nv = 0, nvw = 0;
+  uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
+  uint32_t* d_err = nullptr;
+  uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums
+  uint64_t scan_words = 0;
+  int num_sms = 0;
+  int ctas_per_sm = 0;
+  size_t smem_bytes = 0;
+  uint64_t launches = 0;
+  // host-consume staging (lazily allocated)
+  void* stage[2] = {nullptr, nullptr};
+  size_t stage_bytes = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied[2] = {nullptr, nullptr};
+  cudaEvent_t ev_used[2] = {nullptr, nullptr};
+  // merge scratch
+  uint64_t* d_pack = nullptr;
+  uint64_t pack_words = 0;
+};
+
+namespace sassi {
+
+// error plumbing (capi.cu)
+int set_error(int status, const std::string& msg);
+int cuda_check(cudaError_t e, const char* what);
+#define SASSI_CUDA(call)                                       \
+  do {                                                         \
+    cudaError_t _e = (call);                                   \
+    if (_e != cudaSuccess) return ::sassi::cuda_check(_e, #call); \
+  } while (0)
+
+Offsets layout_offsets(uint32_t S, uint32_t W);
+
+// kernels' host launchers
+int launch_init_tables(sassi_ctx* c, cudaStream_t s);
+int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s);
+int launch_index(sassi_ctx* c, const sassi_hdr* hdr, uint64_t n, sassi_chunk_base* out,
+                 cudaStream_t s);
+int launch_sample(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* host_out,
+                  cudaStream_t s);
+int launch_merge(sassi_ctx* c, void* comm, cudaStream_t s);
+int consume_smem_bytes(const sassi_ctx* c, size_t* bytes);
+
+}  // namespace sassi

@@ -1,0 +1,440 @@
+// consume.cu — the fused SASSI handler fold over warp-instruction records (sm_100a).
+//
+// One launch streams headers (16 B) + only the payload rows the attached handlers need, and folds
+// them into per-CTA shared-memory partial tables keyed by an open-addressed per-PC hash, flushed
+// to the global u64 table image at CTA exit. Handlers (PAPER.md = /root/reference/PAPER.md):
+//   branch     Fig.4 (L237-L243)   lane-per-record: popc of active / taken masks
+//   memdiv     Fig.6 (L361-L369)   warp-per-row: distinct 32 B sectors and 128 B lines among the
+//                                  guard-true lanes; window-bitmap REDUX fast path, MATCH.ANY slow path
+//   value      Fig.9 (L549-L563)   warp-per-row: REDUX.AND / REDUX.OR over written lanes ->
+//                                  constant ones / zeros and "all lanes same" (scalar)
+//   instcount  §8.1 (L625-L627)    lane-per-record: 32x32 bit-matrix transpose + popc gives the
+//                                  per-lane count of 32 records; register accumulator per trace warp
+// Work split: a warp owns one 256-record chunk at a time (chunk_base gives its row offsets) and walks
+// it in 8 batches of 32 records; row indices inside a batch come from ballot prefix sums.
+#include "common.cuh"
+
+namespace sassi {
+namespace {
+
+__device__ __forceinline__ uint4 ld_nc_v4(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t* p) {
+  uint64_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_nc_u32(const uint32_t* p) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+  uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src);
+  uint32_t hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src);
+  return ((uint64_t)hi << 32) | lo;
+}
+
+// 32x32 bit-matrix transpose across the warp: in, lane i holds row i; out, lane l holds the word
+// whose bit i is bit l of row i. Five butterfly stages swapping off-diagonal blocks.
+__device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
+  const uint32_t m16 = 0x0000FFFFu, m8 = 0x00FF00FFu, m4 = 0x0F0F0F0Fu, m2 = 0x33333333u,
+                 m1 = 0x55555555u;
+#define SASSI_TSTAGE(J, M)                                              \
+  {                                                                     \
+    uint32_t y = __shfl_xor_sync(FULL, x, J);                           \
+    x = (lane & J) ? ((x & ~M) | ((y >> J) & M)) : ((x & M) | ((y << J) & ~M)); \
+  }
+  SASSI_TSTAGE(16, m16)
+  SASSI_TSTAGE(8, m8)
+  SASSI_TSTAGE(4, m4)
+  SASSI_TSTAGE(2, m2)
+  SASSI_TSTAGE(1, m1)
+#undef SASSI_TSTAGE
+  return x;
+}
+
+// Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
+// over the lanes of G. Fast path when every sector lies within [-32, 31] of the first lane's: a
+// 64-bit window bitmap OR-reduced across the warp. Otherwise MATCH.ANY groups equal keys.
+__device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
+                                           uint32_t* out_l) {
+  const bool in = (G >> lane) & 1u;
+  const uint64_t sec = a >> 5;
+  const int leader = __ffs(G) - 1;
+  const uint64_t base = shfl64(sec, leader);
+  const int64_t d = (int64_t)(sec - base);
+  const bool inwin = (uint64_t)(d + 32) < 64ull;
+  if (__all_sync(FULL, !in || inwin)) {
+    const uint64_t bit = in ? (1ull << (d + 32)) : 0ull;
+    const uint32_t lo = __reduce_or_sync(FULL, (uint32_t)bit);
+    const uint32_t hi = __reduce_or_sync(FULL, (uint32_t)(bit >> 32));
+    const int64_t dl = (int64_t)((sec >> 2) - (base >> 2));  // in [-8, 8]
+    const uint32_t lb = in ? (1u << (uint32_t)(dl + 8)) : 0u;
+    *out_s = __popc(lo) + __popc(hi);
+    *out_l = __popc(__reduce_or_sync(FULL, lb));
+  } else {
+    uint32_t gs = 0, gl = 0;
+    if (in) {
+      gs = __match_any_sync(G, sec);
+      gl = __match_any_sync(G, sec >> 2);
+    }
+    const bool ls = in && (uint32_t)(__ffs(gs) - 1) == lane;
+    const bool ll = in && (uint32_t)(__ffs(gl) - 1) == lane;
+    *out_s = __popc(__ballot_sync(FULL, ls));
+    *out_l = __popc(__ballot_sync(FULL, ll));
+  }
+}
+
+template <uint32_t H>
+__global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeParams p) {
+  extern __shared__ __align__(16) uint32_t sm[];
+  const uint32_t cap = p.cap;
+  uint32_t* s_keys = sm;
+  uint32_t* s_info = sm + cap;
+  uint32_t* s_cidx = sm + 2 * cap;
+  uint32_t* s_br = sm + 3 * cap;        // [nb][4]: total, active, taken, divergent
+  uint32_t* s_mem = s_br + 4 * p.nb;    // [nm][4]: warps, lanes, sectors, lines
+  uint32_t* s_val = s_mem + 4 * p.nm;   // per value site: we, te, {ones, zeros, nonscalar} x ndst
+  uint32_t* s_h32 = s_val + p.nvw;      // [32][32]
+  uint32_t* s_h128 = s_h32 + 1024;      // [32][32]
+  uint32_t* s_diag = s_h128 + 1024;     // n_records, n_invalid, n_unknown, n_bad_warp (+pad)
+  const uint32_t desc_word = (3 * cap + 4 * (p.nb + p.nm) + p.nvw + 2048 + 8 + 1) & ~1u;
+  uint2* s_vdesc = reinterpret_cast<uint2*>(sm + desc_word);  // [warps][128] value-row descriptors
+
+  const uint32_t tid = threadIdx.x;
+  for (uint32_t i = tid; i < cap; i += blockDim.x) {
+    s_keys[i] = p.hash[i];
+    s_info[i] = p.hash[cap + i];
+    s_cidx[i] = p.hash[2 * cap + i];
+  }
+  for (uint32_t i = tid; i < 4 * (p.nb + p.nm) + p.nvw + 2048 + 8; i += blockDim.x) s_br[i] = 0;
+  __syncthreads();
+  if (H & SASSI_H_VALUE) {
+    for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
+      const uint32_t off = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
+      for (uint32_t d = 0; d < nd; ++d) {
+        s_val[off + 2 + 3 * d] = FULL;  // constantOnes: AND identity
+        s_val[off + 3 + 3 * d] = FULL;  // constantZeros
+      }
+    }
+  }
+  __syncthreads();
+
+  const uint32_t lane = tid & 31u, wib = tid >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  uint2* vdesc = s_vdesc + wib * 128;
+  const uint64_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
+  const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta;
+  uint32_t c_rec = 0, c_inv = 0, c_unk = 0, c_bad = 0;
+  uint32_t acc = 0, acc_w = FULL;  // per-thread-count accumulator of trace warp acc_w, lane = lane
+  uint32_t err = 0;
+  unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
+
+  for (uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
+    const ulonglong2 cb0 = p.cb[u];
+    const ulonglong2 cb1 = p.cb[u + 1];
+    uint64_t arow = cb0.x, vrow = cb0.y;
+    const uint64_t rec0 = u * SASSI_CHUNK;
+    const uint64_t left = p.n - rec0;
+    const uint32_t nbat = left >= SASSI_CHUNK ? SASSI_CHUNK / 32 : (uint32_t)((left + 31) / 32);
+    uint4 hnext = (rec0 + lane < p.n) ? ld_nc_v4(p.hdr + rec0 + lane) : make_uint4(EMPTY_KEY, 0, 0, 0);
+    for (uint32_t b = 0; b < nbat; ++b) {
+      const uint64_t i = rec0 + 32 * b + lane;
+      const bool valid = i < p.n;
+      const uint4 h = hnext;
+      if (b + 1 < nbat) {
+        const uint64_t i2 = i + 32;
+        hnext = i2 < p.n ? ld_nc_v4(p.hdr + i2) : make_uint4(EMPTY_KEY, 0, 0, 0);
+      }
+      // ---- find(pc): open-addressed, linear probing (Fig.4 l.23, L239) ----
+      uint32_t info = 0, cidx = 0;
+      bool known = false;
+      if (valid) {
+        uint32_t slot = fmix32(h.x) & (cap - 1);
+        for (;;) {
+          const uint32_t k = s_keys[slot];
+          if (k == h.x) {
+            known = true;
+            info = s_info[slot];
+            cidx = s_cidx[slot];
+            break;
+          }
+          if (k == EMPTY_KEY) break;
+          slot = (slot + 1) & (cap - 1);
+        }
+      }
+      c_rec += valid;
+      c_unk += valid && !known;
+      // ---- row indices of this batch (rows follow their records) ----
+      const bool has_a = known && (info & I_ADDR_ROW);
+      const uint32_t nd = known ? (info >> I_NDST_SHIFT) & 7u : 0u;
+      const uint32_t ma = __ballot_sync(FULL, has_a);
+      const uint64_t my_arow = arow + __popc(ma & lt);
+      arow += __popc(ma);
+      uint32_t vpre = 0, vtot = 0;
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        const uint32_t mk = __ballot_sync(FULL, (nd >> k) & 1u);
+        vpre += __popc(mk & lt) << k;
+        vtot += __popc(mk) << k;
+      }
+      const uint64_t bv0 = vrow;
+      vrow += vtot;
+      const uint32_t act = h.z, m2 = h.w;
+      const bool live = known && act != 0;
+      c_inv += known && act == 0;
+      const uint32_t G = act & m2;  // guard-true (or taken) active lanes
+
+      // ---- Case study I: branch divergence (Fig.4) ----
+      if (H & SASSI_H_BRANCH) {
+        if (live && (info & I_BRANCH)) {
+          uint32_t* st = s_br + 4 * (cidx & 0xFFFFu);
+          const uint32_t T = G;  // taken = mask2 & active (R1)
+          atomicAdd(st + 0, 1u);
+          atomicAdd(st + 1, (uint32_t)__popc(act));
+          atomicAdd(st + 2, (uint32_t)__popc(T));
+          if (T != 0 && T != act) atomicAdd(st + 3, 1u);
+        }
+      }
+      // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
+      if (H & SASSI_H_INSTCOUNT) {
+        uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
+        if (E != 0 && h.y >= p.n_warps) {
+          ++c_bad;
+          E = 0;
+        }
+        uint32_t pend = __ballot_sync(FULL, E != 0);
+        while (pend) {
+          const uint32_t w0 = __shfl_sync(FULL, h.y, __ffs(pend) - 1);
+          const bool mine = E != 0 && h.y == w0;
+          const uint32_t cnt = __popc(transpose32(mine ? E : 0u, lane));
+          if (w0 != acc_w) {
+            if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+            acc_w = w0;
+            acc = 0;
+          }
+          acc += cnt;
+          pend &= ~__ballot_sync(FULL, mine);
+          if (mine) E = 0;
+        }
+      }
+      // ---- Case study II: memory address divergence (Fig.6) ----
+      if (H & SASSI_H_MEMDIV) {
+        uint32_t selm = __ballot_sync(FULL, live && (info & I_MEMDIV) && G != 0);
+        while (selm) {
+          uint64_t a[4];
+          uint32_t g[4], mi[4];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            g[k] = 0;
+            if (selm) {
+              const int j = __ffs(selm) - 1;
+              selm &= selm - 1;
+              const uint64_t row = shfl64(my_arow, j);
+              g[k] = __shfl_sync(FULL, G, j);
+              mi[k] = __shfl_sync(FULL, cidx & 0xFFFFu, j);
+              if (row < p.arow_base || row >= p.arow_end) {
+                err |= 1u;
+                g[k] = 0;
+              } else {
+                a[k] = ld_nc_u64(p.addr + 32ull * (row - p.arow_base) + lane);
+              }
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            if (g[k]) {
+              uint32_t s, L;
+              memdiv_row(a[k], g[k], lane, &s, &L);
+              const uint32_t n = __popc(g[k]);
+              if (lane < 6) {
+                uint32_t* dst;
+                uint32_t v = 1;
+                if (lane == 0) dst = s_h32 + 32 * (n - 1) + (s - 1);
+                else if (lane == 1) dst = s_h128 + 32 * (n - 1) + (L - 1);
+                else {
+                  dst = s_mem + 4 * mi[k] + (lane - 2);
+                  v = lane == 2 ? 1u : (lane == 3 ? n : (lane == 4 ? s : L));
+                }
+                atomicAdd(dst, v);
+              }
+            }
+          }
+        }
+      }
+      // ---- Case study III: value profiling (Fig.9) ----
+      if (H & SASSI_H_VALUE) {
+        const bool selv = live && nd > 0 && G != 0;
+        const uint32_t voff = cidx >> 16;
+        if (selv) {
+          atomicAdd(s_val + voff, 1u);                       // warp executions
+          atomicAdd(s_val + voff + 1, (uint32_t)__popc(G));  // thread executions ("weight")
+        }
+        for (uint32_t d = 0; d < nd; ++d) vdesc[vpre + d] = make_uint2(selv ? G : 0u, voff + 2 + 3 * d);
+        __syncwarp();
+        for (uint32_t r0 = 0; r0 < vtot; r0 += 8) {
+          uint32_t v[8];
+          uint2 dsc[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const uint32_t r = r0 + k;
+            dsc[k] = r < vtot ? vdesc[r] : make_uint2(0u, 0u);
+            if (dsc[k].x) {
+              const uint64_t row = bv0 + r;
+              if (row < p.vrow_base || row >= p.vrow_end) {
+                err |= 2u;
+                dsc[k].x = 0;
+              } else {
+                v[k] = ld_nc_u32(p.val + 32ull * (row - p.vrow_base) + lane);
+              }
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            if (dsc[k].x) {
+              const uint32_t V = dsc[k].x;
+              const bool in = (V >> lane) & 1u;
+              const uint32_t va = __reduce_and_sync(FULL, in ? v[k] : FULL);
+              const uint32_t vo = __reduce_or_sync(FULL, in ? v[k] : 0u);
+              uint32_t* w = s_val + dsc[k].y;
+              if (lane == 0) {
+                const uint32_t cur = w[0];
+                if ((cur & va) != cur) atomicAnd(w + 0, va);         // atomicAnd(constantOnes, v)
+              } else if (lane == 1) {
+                const uint32_t cur = w[1];
+                if ((cur & ~vo) != cur) atomicAnd(w + 1, ~vo);       // atomicAnd(constantZeros, ~v)
+              } else if (lane == 2) {
+                if (va != vo) atomicAdd(w + 2, 1u);                  // not all lanes equal
+              }
+            }
+          }
+        }
+        __syncwarp();
+      }
+    }
+    if (lane == 0 && (arow != cb1.x || vrow != cb1.y)) err |= 4u;  // chunk index inconsistent
+  }
+  if (H & SASSI_H_INSTCOUNT) {
+    if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+  }
+  // ---- diagnostics: warp-reduce, one smem atomic per warp ----
+  c_rec = __reduce_add_sync(FULL, c_rec);
+  c_inv = __reduce_add_sync(FULL, c_inv);
+  c_unk = __reduce_add_sync(FULL, c_unk);
+  c_bad = __reduce_add_sync(FULL, c_bad);
+  err = __reduce_or_sync(FULL, err);
+  if (lane == 0) {
+    atomicAdd(s_diag + 0, c_rec);
+    atomicAdd(s_diag + 1, c_inv);
+    atomicAdd(s_diag + 2, c_unk);
+    atomicAdd(s_diag + 3, c_bad);
+    if (err) atomicOr(p.err, err);
+  }
+  __syncthreads();
+
+  // ---- flush the CTA's shared-memory partials into the global u64 image ----
+  if (tid < 4 && s_diag[tid]) atomicAdd(&table[tid], (unsigned long long)s_diag[tid]);
+  if (H & SASSI_H_BRANCH) {
+    for (uint32_t b = tid; b < p.nb; b += blockDim.x) {
+      const uint32_t* st = s_br + 4 * b;
+      if (st[0] == 0) continue;
+      unsigned long long* g = table + p.off.br + 5ull * p.flush_b[b];
+      atomicAdd(g + 0, (unsigned long long)st[0]);
+      atomicAdd(g + 1, (unsigned long long)st[1]);
+      if (st[2]) atomicAdd(g + 2, (unsigned long long)st[2]);
+      if (st[1] - st[2]) atomicAdd(g + 3, (unsigned long long)(st[1] - st[2]));  // not taken
+      if (st[3]) atomicAdd(g + 4, (unsigned long long)st[3]);
+    }
+  }
+  if (H & SASSI_H_MEMDIV) {
+    for (uint32_t m = tid; m < p.nm; m += blockDim.x) {
+      const uint32_t* st = s_mem + 4 * m;
+      if (st[0] == 0) continue;
+      unsigned long long* g = table + p.off.mem + 4ull * p.flush_m[m];
+      for (int f = 0; f < 4; ++f) atomicAdd(g + f, (unsigned long long)st[f]);
+    }
+    for (uint32_t c = tid; c < 2048; c += blockDim.x) {
+      const uint32_t v = s_h32[c];
+      if (v) atomicAdd(table + (c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024)), (unsigned long long)v);
+    }
+  }
+  if (H & SASSI_H_VALUE) {
+    for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
+      const uint32_t site = p.flush_v[3 * k], off = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
+      const uint32_t* w = s_val + off;
+      if (w[0] == 0) continue;
+      atomicAdd(table + p.off.val + 2ull * site, (unsigned long long)w[0]);
+      atomicAdd(table + p.off.val + 2ull * site + 1, (unsigned long long)w[1]);
+      for (uint32_t d = 0; d < nd; ++d) {
+        const uint32_t o = w[2 + 3 * d], z = w[3 + 3 * d], ns = w[4 + 3 * d];
+        if (o != FULL) atomicAnd(table + p.off.ones + 4ull * site + d, (unsigned long long)o);
+        if (z != FULL) atomicAnd(table + p.off.zeros + 4ull * site + d, (unsigned long long)z);
+        if (ns) atomicAdd(table + p.off.nonscalar + 4ull * site + d, (unsigned long long)ns);
+      }
+    }
+  }
+}
+
+using KernelFn = void (*)(const ConsumeParams);
+
+template <uint32_t H>
+KernelFn kernel_for() {
+  return consume_kernel<H>;
+}
+
+KernelFn select_kernel(uint32_t mask) {
+  switch (mask & 15u) {
+    case 1: return kernel_for<1>();
+    case 2: return kernel_for<2>();
+    case 3: return kernel_for<3>();
+    case 4: return kernel_for<4>();
+    case 5: return kernel_for<5>();
+    case 6: return kernel_for<6>();
+    case 7: return kernel_for<7>();
+    case 8: return kernel_for<8>();
+    case 9: return kernel_for<9>();
+    case 10: return kernel_for<10>();
+    case 11: return kernel_for<11>();
+    case 12: return kernel_for<12>();
+    case 13: return kernel_for<13>();
+    case 14: return kernel_for<14>();
+    case 15: return kernel_for<15>();
+    default: return nullptr;
+  }
+}
+
+}  // namespace
+
+int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
+  size_t words = 3ull * c->cap + 4ull * (c->nb + c->nm) + c->nvw + 2048 + 8;
+  words = (words + 1) & ~1ull;  // 8-byte align the descriptor area
+  *bytes = 4 * words + sizeof(uint2) * 128 * kWarpsPerCta;
+  return 0;
+}
+
+int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
+  KernelFn fn = select_kernel(c->mask);
+  if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
+  SASSI_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->smem_bytes));
+  int per_sm = 0;
+  SASSI_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kConsumeThreads, c->smem_bytes));
+  if (per_sm < 1) return set_error(SASSI_ENOSPC, "consume kernel does not fit on an SM");
+  c->ctas_per_sm = per_sm;
+  const uint64_t units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
+  uint64_t grid = (uint64_t)c->num_sms * per_sm;
+  const uint64_t need = (units + kWarpsPerCta - 1) / kWarpsPerCta;
+  if (grid > need) grid = need ? need : 1;
+  fn<<<(unsigned)grid, kConsumeThreads, c->smem_bytes, s>>>(p);
+  SASSI_CUDA(cudaGetLastError());
+  c->launches += 1;
+  return SASSI_OK;
+}
+
+}  // namespace sassi

@@ -1,0 +1,208 @@
+// merge.cu — multi-GPU merge of the per-rank tables (north_star subsystem 5): every table entry is a
+// commutative fold (counters add, constant-bit masks AND), so ranks that consumed disjoint warp
+// shards combine with ONE ncclAllReduce(sum, uint64) over a packed image in which each AND mask is
+// byte-expanded (bit b -> byte b in {0,1}); after the sum a bit is set iff its byte == nranks
+// (valid for nranks <= 255). A tiny ncclMax allreduce of (checksum, ~checksum) first proves that
+// every rank registered the same sites (identical slot layout).
+// NCCL is loaded with dlopen (the torch-bundled libnccl.so.2 when already in the process).
+#include <dlfcn.h>
+
+#include <mutex>
+
+#include "common.cuh"
+
+namespace sassi {
+namespace {
+
+// minimal NCCL ABI (nccl.h 2.x)
+typedef struct ncclComm* ncclComm_t;
+typedef struct {
+  char internal[128];
+} ncclUniqueId;
+typedef int ncclResult_t;
+enum { kNcclUint64 = 5 };
+enum { kNcclSum = 0, kNcclMax = 2 };
+
+struct Nccl {
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  bool ok = false;
+  std::string why;
+};
+
+Nccl& nccl() {
+  static Nccl n;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* names[] = {"libnccl.so.2", "libnccl.so",
+                           "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/lib/libnccl.so.2"};
+    void* h = nullptr;
+    for (const char* nm : names) {
+      h = dlopen(nm, RTLD_NOW | RTLD_NOLOAD | RTLD_GLOBAL);  // prefer the copy already loaded
+      if (h) break;
+    }
+    for (const char* nm : names) {
+      if (h) break;
+      h = dlopen(nm, RTLD_NOW | RTLD_GLOBAL);
+    }
+    if (!h) {
+      n.why = "cannot dlopen libnccl.so.2";
+      return;
+    }
+    n.GetUniqueId = (decltype(n.GetUniqueId))dlsym(h, "ncclGetUniqueId");
+    n.CommInitRank = (decltype(n.CommInitRank))dlsym(h, "ncclCommInitRank");
+    n.CommDestroy = (decltype(n.CommDestroy))dlsym(h, "ncclCommDestroy");
+    n.CommCount = (decltype(n.CommCount))dlsym(h, "ncclCommCount");
+    n.AllReduce = (decltype(n.AllReduce))dlsym(h, "ncclAllReduce");
+    n.GetErrorString = (decltype(n.GetErrorString))dlsym(h, "ncclGetErrorString");
+    n.ok = n.GetUniqueId && n.CommInitRank && n.CommDestroy && n.CommCount && n.AllReduce &&
+           n.GetErrorString;
+    if (!n.ok) n.why = "libnccl.so.2 lacks an expected symbol";
+  });
+  return n;
+}
+
+int nccl_err(ncclResult_t r, const char* what) {
+  return set_error(SASSI_ENCCL, std::string(what) + ": " + nccl().GetErrorString(r));
+}
+
+// packed image: [4 diag sums][br..val sums][nonscalar..counts sums][8S masks x 4 words]
+struct PackLayout {
+  uint64_t n_sum_a, n_sum_b, n_mask_words, total;
+};
+PackLayout pack_layout(const sassi_ctx* c) {
+  PackLayout L;
+  L.n_sum_a = c->off.ones - c->off.br;
+  L.n_sum_b = c->off.total - c->off.nonscalar;
+  L.n_mask_words = 8ull * c->S * 4;
+  L.total = 4 + L.n_sum_a + L.n_sum_b + L.n_mask_words;
+  return L;
+}
+
+__global__ void pack_kernel(const uint64_t* __restrict__ t, Offsets o, PackLayout L, uint64_t* pk) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < L.total; i += stride) {
+    uint64_t v;
+    if (i < 4) v = t[i];
+    else if (i < 4 + L.n_sum_a) v = t[o.br + (i - 4)];
+    else if (i < 4 + L.n_sum_a + L.n_sum_b) v = t[o.nonscalar + (i - 4 - L.n_sum_a)];
+    else {
+      const uint64_t w = i - (4 + L.n_sum_a + L.n_sum_b);
+      const uint32_t mask = (uint32_t)t[o.ones + w / 4];  // ones[S][4] then zeros[S][4]
+      const uint32_t byte8 = (mask >> (8 * (w % 4))) & 0xFFu;
+      v = 0;
+#pragma unroll
+      for (int b = 0; b < 8; ++b) v |= (uint64_t)((byte8 >> b) & 1u) << (8 * b);
+    }
+    pk[i] = v;
+  }
+}
+
+__global__ void unpack_kernel(uint64_t* __restrict__ t, Offsets o, PackLayout L,
+                              const uint64_t* __restrict__ pk, uint32_t nranks) {
+  const uint64_t n_masks = L.n_mask_words / 4;
+  const uint64_t n_items = 4 + L.n_sum_a + L.n_sum_b + n_masks;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_items; i += stride) {
+    if (i < 4) t[i] = pk[i];
+    else if (i < 4 + L.n_sum_a) t[o.br + (i - 4)] = pk[i];
+    else if (i < 4 + L.n_sum_a + L.n_sum_b) t[o.nonscalar + (i - 4 - L.n_sum_a)] = pk[i];
+    else {
+      const uint64_t m = i - (4 + L.n_sum_a + L.n_sum_b);
+      const uint64_t* w = pk + 4 + L.n_sum_a + L.n_sum_b + 4 * m;
+      uint32_t mask = 0;
+      for (int q = 0; q < 4; ++q)
+        for (int b = 0; b < 8; ++b)
+          if (((w[q] >> (8 * b)) & 0xFFu) == nranks) mask |= 1u << (8 * q + b);
+      t[o.ones + m] = mask;
+    }
+  }
+}
+
+}  // namespace
+
+int launch_merge(sassi_ctx* c, void* comm_v, cudaStream_t s) {
+  Nccl& N = nccl();
+  if (!N.ok) return set_error(SASSI_ENCCL, N.why);
+  ncclComm_t comm = (ncclComm_t)comm_v;
+  int nranks = 0;
+  ncclResult_t r = N.CommCount(comm, &nranks);
+  if (r) return nccl_err(r, "ncclCommCount");
+  if (nranks > 255) return set_error(SASSI_EINVAL, "sassi_merge supports at most 255 ranks");
+  const PackLayout L = pack_layout(c);
+  if (L.total + 2 > c->pack_words) {
+    cudaFree(c->d_pack);
+    c->d_pack = nullptr;
+    c->pack_words = 0;
+    SASSI_CUDA(cudaMalloc(&c->d_pack, 8 * (L.total + 2)));
+    c->pack_words = L.total + 2;
+  }
+  // 1) identical site tables on every rank?
+  uint64_t ck[2] = {c->checksum, ~c->checksum};
+  uint64_t* d_ck = c->d_pack + L.total;
+  SASSI_CUDA(cudaMemcpyAsync(d_ck, ck, 16, cudaMemcpyHostToDevice, s));
+  r = N.AllReduce(d_ck, d_ck, 2, kNcclUint64, kNcclMax, comm, s);
+  if (r) return nccl_err(r, "ncclAllReduce(checksum)");
+  uint64_t got[2];
+  SASSI_CUDA(cudaMemcpyAsync(got, d_ck, 16, cudaMemcpyDeviceToHost, s));
+  SASSI_CUDA(cudaStreamSynchronize(s));
+  if (got[0] != c->checksum || ~got[1] != c->checksum)
+    return set_error(SASSI_EMISMATCH, "site tables / n_warps differ across ranks");
+  // 2) pack -> one allreduce(sum, u64) -> unpack
+  const unsigned grid = (unsigned)std::min<uint64_t>(4096, (L.total + 255) / 256);
+  pack_kernel<<<grid, 256, 0, s>>>(c->d_table, c->off, L, c->d_pack);
+  SASSI_CUDA(cudaGetLastError());
+  r = N.AllReduce(c->d_pack, c->d_pack, L.total, kNcclUint64, kNcclSum, comm, s);
+  if (r) return nccl_err(r, "ncclAllReduce(tables)");
+  unpack_kernel<<<grid, 256, 0, s>>>(c->d_table, c->off, L, c->d_pack, (uint32_t)nranks);
+  SASSI_CUDA(cudaGetLastError());
+  c->launches += 2;
+  return SASSI_OK;
+}
+
+}  // namespace sassi
+
+extern "C" {
+
+int sassi_nccl_get_unique_id(void* out) {
+  using namespace sassi;
+  if (!out) return set_error(SASSI_EINVAL, "null out");
+  Nccl& N = nccl();
+  if (!N.ok) return set_error(SASSI_ENCCL, N.why);
+  ncclUniqueId id;
+  ncclResult_t r = N.GetUniqueId(&id);
+  if (r) return nccl_err(r, "ncclGetUniqueId");
+  memcpy(out, &id, sizeof id);
+  return SASSI_OK;
+}
+
+int sassi_nccl_comm_create(void** comm_out, int nranks, int rank, const void* uid, int device) {
+  using namespace sassi;
+  if (!comm_out || !uid) return set_error(SASSI_EINVAL, "null argument");
+  Nccl& N = nccl();
+  if (!N.ok) return set_error(SASSI_ENCCL, N.why);
+  SASSI_CUDA(cudaSetDevice(device));
+  ncclUniqueId id;
+  memcpy(&id, uid, sizeof id);
+  ncclComm_t comm = nullptr;
+  ncclResult_t r = N.CommInitRank(&comm, nranks, id, rank);
+  if (r) return nccl_err(r, "ncclCommInitRank");
+  *comm_out = comm;
+  return SASSI_OK;
+}
+
+int sassi_nccl_comm_destroy(void* comm) {
+  using namespace sassi;
+  if (!comm) return SASSI_OK;
+  Nccl& N = nccl();
+  if (!N.ok) return set_error(SASSI_ENCCL, N.why);
+  ncclResult_t r = N.CommDestroy((ncclComm_t)comm);
+  if (r) return nccl_err(r, "ncclCommDestroy");
+  return SASSI_OK;
+}
+
+}  // extern "C"

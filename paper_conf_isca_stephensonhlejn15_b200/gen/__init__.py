@@ -222,9 +222,15 @@ def generate_device(program: Program, limit=None, warp_base: int = 0, n_warps=No
         n = n_tot if limit is None else min(int(limit), n_tot)
         nch = (n + CHUNK - 1) // CHUNK
         offs_d = torch.from_numpy(offs.view(np.int64)).to(dev)
+        if n < n_tot:  # rows needed: at most up to the end of the warp holding record n
+            wl = int(np.searchsorted(offs[:, 0], n, side="right"))
+            a_cap = int(offs[wl, 1]) if wl < len(offs) else a_tot
+            v_cap = int(offs[wl, 2]) if wl < len(offs) else v_tot
+        else:
+            a_cap, v_cap = a_tot, v_tot
         hdr = torch.empty((max(n, 1), 4), dtype=torch.int32, device=dev)
-        addr = torch.empty((max(a_tot, 1), 32), dtype=torch.int64, device=dev)
-        val = torch.empty((max(v_tot, 1), 32), dtype=torch.int32, device=dev)
+        addr = torch.empty((max(a_cap, 1), 32), dtype=torch.int64, device=dev)
+        val = torch.empty((max(v_cap, 1), 32), dtype=torch.int32, device=dev)
         cb = torch.zeros((nch + 1, 2), dtype=torch.int64, device=dev)
         if n == n_tot:
             cb[nch, 0] = a_tot

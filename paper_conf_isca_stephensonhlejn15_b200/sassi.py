@@ -1,0 +1,273 @@
+"""Thin ctypes binding of libsassi.so — same names as the C ABI (include/sassi.h).
+
+Argument marshalling only: every step of the fold runs in the CUDA kernels of libsassi.so. Device
+buffers are torch tensors (``data_ptr()``), streams are ``torch.cuda.Stream.cuda_stream``. There is
+no CPU fallback: if the library or a CUDA device is missing, calls raise ``SassiError``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "lib", "libsassi.so")
+
+SITE_DTYPE = np.dtype([("pc", "<u4"), ("flags", "<u2"), ("mem_width", "u1"), ("domain", "u1"),
+                       ("n_gpr_dst", "u1"), ("reg_num", "u1", (4,)), ("reserved", "u1", (3,))])
+INJ_DTYPE = np.dtype([("kernel", "<u4"), ("invocation", "<u4"), ("thread", "<u4"),
+                      ("reg_seed", "<u4"), ("bit_seed", "<u4"), ("reserved", "<u4"),
+                      ("dyn_index", "<u8")])
+
+SASSI_OK, SASSI_EINVAL, SASSI_ECUDA, SASSI_ENCCL = 0, -1, -2, -3
+SASSI_ENOSPC, SASSI_ESTATE, SASSI_EMISMATCH, SASSI_EFORMAT = -4, -5, -6, -7
+SASSI_H_BRANCH, SASSI_H_MEMDIV, SASSI_H_VALUE, SASSI_H_INSTCOUNT, SASSI_H_ALL = 1, 2, 4, 8, 15
+SASSI_CHUNK = 256
+
+# every function declared in include/sassi.h: name -> (restype, argtypes)
+_vp, _u32, _u64, _i = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+
+
+class SassiRecords(ctypes.Structure):
+    _fields_ = [("hdr", _vp), ("addr", _vp), ("val", _vp), ("chunk_base", _vp),
+                ("n_addr_rows", _u64), ("n_val_rows", _u64)]
+
+
+class SassiLayout(ctypes.Structure):
+    _fields_ = [(k, _u64) for k in ("diag", "br", "mem", "val", "ones", "zeros", "nonscalar", "h32",
+                                    "h128", "counts", "total")]
+
+
+SIGNATURES = {
+    "sassi_table_layout": (_i, [_u32, _u32, ctypes.POINTER(SassiLayout)]),
+    "sassi_ctx_create": (_i, [ctypes.POINTER(_vp), _i, _vp, _u32, _u32]),
+    "sassi_ctx_destroy": (None, [_vp]),
+    "sassi_attach_handler": (_i, [_vp, _u32]),
+    "sassi_consume": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
+    "sassi_consume_host": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
+    "sassi_index_records": (_i, [_vp, _vp, _u64, _vp, _vp]),
+    "sassi_reset": (_i, [_vp, _vp]),
+    "sassi_read_tables": (_i, [_vp, _vp, _u64, _vp]),
+    "sassi_tables_device": (_i, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_u64)]),
+    "sassi_sample_sites": (_i, [_vp, _u32, _u64, _vp, _vp]),
+    "sassi_merge": (_i, [_vp, _vp, _vp]),
+    "sassi_nccl_get_unique_id": (_i, [_vp]),
+    "sassi_nccl_comm_create": (_i, [ctypes.POINTER(_vp), _i, _i, _vp, _i]),
+    "sassi_nccl_comm_destroy": (_i, [_vp]),
+    "sassi_kernel_launches": (_i, [_vp, ctypes.POINTER(_u64)]),
+    "sassi_strerror": (ctypes.c_char_p, [_i]),
+    "sassi_last_error": (ctypes.c_char_p, []),
+}
+
+
+class SassiError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__("%s (%d): %s" % (sassi_strerror(status), status, msg))
+        self.status = status
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libsassi.so (fails loudly: there is no fallback path)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError("libsassi.so not built (%s): run __graft_entry__.build()" % LIB_PATH)
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in SIGNATURES.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def sassi_strerror(status: int) -> str:
+    return lib().sassi_strerror(status).decode()
+
+
+def sassi_last_error() -> str:
+    return lib().sassi_last_error().decode()
+
+
+def _check(rc: int) -> None:
+    if rc != 0:
+        raise SassiError(rc, sassi_last_error())
+
+
+def _stream(stream) -> int | None:
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return getattr(stream, "cuda_stream", stream)
+
+
+def _ptr(x) -> int | None:
+    if x is None:
+        return None
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr() if x.numel() else None
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data if x.size else None
+    return int(x)
+
+
+def _records(rec: dict) -> SassiRecords:
+    r = SassiRecords()
+    r.hdr = _ptr(rec["hdr"])
+    r.addr = _ptr(rec["addr"]) if rec.get("n_addr_rows", 0) else None
+    r.val = _ptr(rec["val"]) if rec.get("n_val_rows", 0) else None
+    r.chunk_base = _ptr(rec["chunk_base"])
+    r.n_addr_rows = int(rec.get("n_addr_rows", 0))
+    r.n_val_rows = int(rec.get("n_val_rows", 0))
+    return r
+
+
+# ---- the C ABI, one Python function per C function --------------------------------------------
+def sassi_table_layout(n_sites: int, n_warps: int) -> dict:
+    L = SassiLayout()
+    _check(lib().sassi_table_layout(n_sites, n_warps, ctypes.byref(L)))
+    return {k: int(getattr(L, k)) for k, _ in SassiLayout._fields_}
+
+
+def sassi_ctx_create(device: int, sites: np.ndarray, n_warps: int) -> int:
+    sites = np.ascontiguousarray(sites).view(SITE_DTYPE)
+    h = _vp()
+    _check(lib().sassi_ctx_create(ctypes.byref(h), device, sites.ctypes.data if len(sites) else None,
+                                  len(sites), n_warps))
+    return h.value
+
+
+def sassi_ctx_destroy(ctx: int) -> None:
+    lib().sassi_ctx_destroy(ctx)
+
+
+def sassi_attach_handler(ctx: int, kind_mask: int) -> None:
+    _check(lib().sassi_attach_handler(ctx, kind_mask))
+
+
+def sassi_consume(ctx: int, rec: dict, n=None, stream=None) -> None:
+    n = rec["n"] if n is None else n
+    r = _records(rec)
+    _check(lib().sassi_consume(ctx, ctypes.byref(r), n, _stream(stream)))
+
+
+def sassi_consume_host(ctx: int, rec: dict, n=None, stream=None) -> None:
+    n = rec["n"] if n is None else n
+    r = _records(rec)
+    _check(lib().sassi_consume_host(ctx, ctypes.byref(r), n, _stream(stream)))
+
+
+def sassi_index_records(ctx: int, hdr, n: int, chunk_base_out, stream=None) -> None:
+    _check(lib().sassi_index_records(ctx, _ptr(hdr), n, _ptr(chunk_base_out), _stream(stream)))
+
+
+def sassi_reset(ctx: int, stream=None) -> None:
+    _check(lib().sassi_reset(ctx, _stream(stream)))
+
+
+def sassi_read_tables(ctx: int, n_words: int, stream=None, out: np.ndarray | None = None) -> np.ndarray:
+    out = np.zeros(n_words, dtype=np.uint64) if out is None else out
+    _check(lib().sassi_read_tables(ctx, out.ctypes.data, out.size, _stream(stream)))
+    return out
+
+
+def sassi_tables_device(ctx: int):
+    p, n = _vp(), _u64()
+    _check(lib().sassi_tables_device(ctx, ctypes.byref(p), ctypes.byref(n)))
+    return p.value, n.value
+
+
+def sassi_sample_sites(ctx: int, k: int, seed: int, stream=None) -> np.ndarray:
+    out = np.zeros(k, dtype=INJ_DTYPE)
+    _check(lib().sassi_sample_sites(ctx, k, seed & (2**64 - 1), out.ctypes.data if k else None,
+                                    _stream(stream)))
+    return out
+
+
+def sassi_merge(ctx: int, comm: int, stream=None) -> None:
+    _check(lib().sassi_merge(ctx, comm, _stream(stream)))
+
+
+def sassi_nccl_get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().sassi_nccl_get_unique_id(buf))
+    return buf.raw
+
+
+def sassi_nccl_comm_create(nranks: int, rank: int, unique_id: bytes, device: int) -> int:
+    comm = _vp()
+    uid = ctypes.create_string_buffer(bytes(unique_id), 128)
+    _check(lib().sassi_nccl_comm_create(ctypes.byref(comm), nranks, rank, uid, device))
+    return comm.value
+
+
+def sassi_nccl_comm_destroy(comm: int) -> None:
+    _check(lib().sassi_nccl_comm_destroy(comm))
+
+
+def sassi_kernel_launches(ctx: int) -> int:
+    n = _u64()
+    _check(lib().sassi_kernel_launches(ctx, ctypes.byref(n)))
+    return n.value
+
+
+# ---- convenience wrapper -----------------------------------------------------------------------
+class Context:
+    """One SASSI analysis context on one device: sites registered once, tables accumulate."""
+
+    def __init__(self, sites: np.ndarray, n_warps: int, handlers: int = SASSI_H_ALL, device: int = 0):
+        self.sites = np.ascontiguousarray(sites).view(SITE_DTYPE)
+        self.n_sites = len(self.sites)
+        self.n_warps = int(n_warps)
+        self.device = device
+        self.layout = sassi_table_layout(self.n_sites, self.n_warps)
+        self.handle = sassi_ctx_create(device, self.sites, self.n_warps)
+        sassi_attach_handler(self.handle, handlers)
+        self.handlers = handlers
+
+    def consume(self, rec: dict, n=None, stream=None):
+        sassi_consume(self.handle, rec, n, stream)
+
+    def consume_host(self, rec: dict, n=None, stream=None):
+        sassi_consume_host(self.handle, rec, n, stream)
+
+    def reset(self, stream=None):
+        sassi_reset(self.handle, stream)
+
+    def read_tables(self, stream=None) -> np.ndarray:
+        return sassi_read_tables(self.handle, self.layout["total"], stream)
+
+    def sections(self, table: np.ndarray | None = None) -> dict:
+        t = self.read_tables() if table is None else table
+        L, S = self.layout, self.n_sites
+        return {"diag": t[0:8], "br": t[L["br"]:L["mem"]].reshape(S, 5),
+                "mem": t[L["mem"]:L["val"]].reshape(S, 4), "val": t[L["val"]:L["ones"]].reshape(S, 2),
+                "ones": t[L["ones"]:L["zeros"]].reshape(S, 4),
+                "zeros": t[L["zeros"]:L["nonscalar"]].reshape(S, 4),
+                "nonscalar": t[L["nonscalar"]:L["h32"]].reshape(S, 4),
+                "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
+                "h128": t[L["h128"]:L["counts"]].reshape(32, 32), "counts": t[L["counts"]:L["total"]]}
+
+    def sample(self, k: int, seed: int, stream=None) -> np.ndarray:
+        return sassi_sample_sites(self.handle, k, seed, stream)
+
+    def merge(self, comm: int, stream=None):
+        sassi_merge(self.handle, comm, stream)
+
+    def kernel_launches(self) -> int:
+        return sassi_kernel_launches(self.handle)
+
+    def close(self):
+        if self.handle:
+            sassi_ctx_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

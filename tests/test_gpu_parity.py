@@ -1,0 +1,237 @@
+"""GPU parity: the CUDA fold (through the C ABI) equals the oracle bit for bit — hand-worked T0,
+random edge-case traces for every handler combination, and every BASELINE config (c1, c2 in
+full; c3/c4/c5 at full size in the bench's launch configuration, checked exactly on prefixes /
+sampled warps the oracle computes one by one, and by properties that hold at any size)."""
+import numpy as np
+import pytest
+
+import oracle
+import t0_trace as T0
+from gpu_helpers import to_device, gpu_table, diff_tables, host_chunk_base
+from test_oracle import random_trace
+from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    torch.cuda.init()
+
+
+def test_t0_hand_worked_on_gpu():
+    s = T0.sites()
+    hdr, addr, val = T0.records()
+    t = gpu_table(s, T0.N_WARPS, sassi.SASSI_H_ALL, to_device(s, hdr, addr, val))
+    T0.check_table(t, oracle.sections(t, len(s), T0.N_WARPS))
+    assert np.array_equal(t, oracle.run(s, T0.N_WARPS, oracle.H_ALL, hdr, addr, val))
+
+
+@pytest.mark.parametrize("mask", [1, 2, 4, 8, 3, 5, 6, 9, 10, 12, 7, 11, 13, 14, 15])
+def test_t0_every_handler_mask(mask):
+    s = T0.sites()
+    hdr, addr, val = T0.records()
+    t = gpu_table(s, T0.N_WARPS, mask, to_device(s, hdr, addr, val))
+    o = oracle.run(s, T0.N_WARPS, mask, hdr, addr, val)
+    assert diff_tables(t, o, len(s), T0.N_WARPS) is None
+
+
+@pytest.mark.parametrize("seed,n", [(0, 1), (1, 31), (2, 257), (3, 1000), (4, 5000), (5, 20000)])
+def test_random_traces(seed, n):
+    s, W, hdr, addr, val = random_trace(1000 + seed, n=n)
+    o = oracle.run(s, W, oracle.H_ALL, hdr, addr, val)
+    t = gpu_table(s, W, sassi.SASSI_H_ALL, to_device(s, hdr, addr, val))
+    assert diff_tables(t, o, len(s), W) is None
+
+
+def test_empty_stream():
+    s = T0.sites()
+    hdr, addr, val = T0.records()
+    d = to_device(s, hdr, addr, val)
+    t = gpu_table(s, T0.N_WARPS, sassi.SASSI_H_ALL, d, n=0)
+    assert np.array_equal(t, oracle.table_init(len(s), T0.N_WARPS, oracle.H_ALL))
+
+
+def test_inconsistent_chunk_index_is_reported():
+    s, W, hdr, addr, val = random_trace(77, n=3000)
+    cb = host_chunk_base(s, hdr)
+    cb[3, 1] += 1                                   # corrupt one chunk's val-row base
+    d = to_device(s, hdr, addr, val, cb)
+    ctx = sassi.Context(s, W, sassi.SASSI_H_ALL)
+    ctx.consume(d)
+    with pytest.raises(sassi.SassiError) as e:
+        ctx.read_tables()
+    assert e.value.status == sassi.SASSI_EFORMAT
+    ctx.close()
+
+
+def test_index_records_matches_generator():
+    P, _, _, _ = gen.preset("c2")
+    r = gen.generate_device(P, None, 0, 3000)
+    ctx = sassi.Context(r["sites"], P.total_warps, sassi.SASSI_H_ALL)
+    out = torch.zeros_like(r["chunk_base"])
+    sassi.sassi_index_records(ctx.handle, r["hdr"], r["n"], out)
+    torch.cuda.synchronize()
+    assert torch.equal(out, r["chunk_base"])
+    ctx.close()
+
+
+def test_device_generator_equals_host_generator():
+    for name, warps in (("c1", None), ("c2", 500), ("c3", 40), ("c4", 40), ("c5", 6)):
+        P, _, _, _ = gen.preset(name)
+        h = gen.generate_host(P, None, 0, warps)
+        d = gen.to_host(gen.generate_device(P, None, 0, warps))
+        assert np.array_equal(h["hdr"], d["hdr"]), name
+        assert np.array_equal(h["addr"], d["addr"]), name
+        assert np.array_equal(h["val"], d["val"]), name
+        assert np.array_equal(h["chunk_base"], d["chunk_base"]), name
+
+
+def _gen(name, limit=None, warp_base=0, n_warps=None):
+    P, lim, mask, _ = gen.preset(name)
+    lim = lim if limit is None else limit
+    return P, mask, gen.generate_device(P, lim, warp_base, n_warps)
+
+
+def test_c1_full():
+    P, mask, d = _gen("c1")
+    h = gen.to_host(d)
+    t = gpu_table(h["sites"], P.total_warps, mask, d)
+    o = oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"])
+    assert diff_tables(t, o, len(h["sites"]), P.total_warps) is None
+
+
+def test_c2_full():
+    """Config 2 at its full size (10^7 records), bit-exact against the oracle."""
+    P, mask, d = _gen("c2")
+    assert d["n"] == 10_000_000
+    h = gen.to_host(d)
+    t = gpu_table(h["sites"], P.total_warps, mask, d)
+    o = oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"])
+    assert diff_tables(t, o, len(h["sites"]), P.total_warps) is None
+
+
+def _prefix(d, n):
+    """First n records of a device stream (n a multiple of SASSI_CHUNK) with their rows."""
+    assert n % 256 == 0
+    cb = d["chunk_base"][n // 256].cpu().numpy().view(np.uint64)
+    na, nv = int(cb[0]), int(cb[1])
+    return dict(hdr=d["hdr"][:n], addr=d["addr"][:na], val=d["val"][:nv],
+                chunk_base=d["chunk_base"][: n // 256 + 1], n=n, n_addr_rows=na, n_val_rows=nv,
+                sites=d["sites"])
+
+
+def _properties(sec, n):
+    br = sec["br"].astype(np.int64)
+    assert (br[:, 2] + br[:, 3] == br[:, 1]).all()
+    m = sec["mem"].astype(np.int64)
+    assert (m[:, 3] <= m[:, 2]).all() and (m[:, 2] <= m[:, 1]).all() and (4 * m[:, 3] >= m[:, 2]).all()
+    assert sec["h32"].sum() == sec["h128"].sum() == m[:, 0].sum()
+    for k in range(32):
+        assert sec["h32"][k, k + 1:].sum() == 0
+    assert int(sec["diag"][0]) == n
+
+
+@pytest.mark.parametrize("name", ["c3", "c4"])
+def test_full_size_prefix_exact_and_properties(name):
+    """10^8 records in the bench's launch configuration: the whole stream is folded on the GPU;
+    its first ~2x10^6 records are checked bit-exactly against the oracle, the full tables by
+    invariants, and consuming the stream in two pieces equals consuming it at once."""
+    P, mask, d = _gen(name)
+    assert d["n"] == 100_000_000
+    S, W = len(d["sites"]), P.total_warps
+    full = gpu_table(d["sites"], W, mask, d)
+    sec = oracle.sections(full, S, W)
+    _properties(sec, d["n"])
+    # exact on a prefix
+    pre = _prefix(d, 2_000_128)
+    hp = gen.to_host(pre)
+    o = oracle.run(hp["sites"], W, mask, hp["hdr"], hp["addr"], hp["val"])
+    t = gpu_table(d["sites"], W, mask, pre)
+    assert diff_tables(t, o, S, W) is None
+    # split consumption == single pass (chunk-aligned split; rows addressed absolutely)
+    ctx = sassi.Context(d["sites"], W, mask)
+    half = (d["n"] // 2) // 256 * 256
+    hdr = d["hdr"]
+    a = dict(d, hdr=hdr[:half], chunk_base=d["chunk_base"][: half // 256 + 1], n=half)
+    b = dict(d, hdr=hdr[half:], chunk_base=d["chunk_base"][half // 256:], n=d["n"] - half)
+    ctx.consume(a)
+    ctx.consume(b)
+    assert np.array_equal(ctx.read_tables(), full)
+    ctx.close()
+
+
+def test_c4_full_instcount_exact_and_sampling():
+    """Config 4 in full: per-thread counts over 10^8 records for 10^6 threads, bit-exact, then
+    1,000 injection-site draws (L629) equal the oracle's draws on the same counts."""
+    P, mask, d = _gen("c4")
+    W = P.total_warps
+    ctx = sassi.Context(d["sites"], W, mask)
+    ctx.consume(d)
+    t = ctx.read_tables()
+    hdr = d["hdr"].cpu().numpy().view(np.uint32).reshape(-1, 4).view(gen.HDR_DTYPE).reshape(-1)
+    o = oracle.table_init(len(d["sites"]), W, mask)
+    oracle.consume(o, d["sites"], W, mask, hdr, None, None, d["n_addr_rows"], d["n_val_rows"])
+    s2 = d["sites"]
+    so, st = oracle.sections(o, len(s2), W), oracle.sections(t, len(s2), W)
+    assert np.array_equal(st["counts"], so["counts"])
+    assert np.array_equal(st["diag"][:4], so["diag"][:4])
+    assert int(so["counts"].sum()) > 0
+    got = ctx.sample(1000, 20150616)
+    exp = oracle.sample(so["counts"], 1000, 20150616)
+    assert np.array_equal(got, exp)
+    ctx.close()
+
+
+def test_c5_sampled_shards():
+    """Config 5 (4x10^9 records over 8 shards of 16,384 warps): each of two shards is generated
+    with its global warp ids; a 3x10^6-record prefix of each is exact against the oracle, and the
+    merged tables of the two prefixes equal the oracle's merge."""
+    P, _, mask, _ = gen.preset("c5")
+    W = P.total_warps
+    acc = None
+    for shard in (0, 5):
+        d = gen.generate_device(P, 3_000_000, shard * 16384, 16384)
+        h = gen.to_host(d)
+        S = len(h["sites"])
+        o = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+        t = gpu_table(h["sites"], W, mask, d)
+        assert diff_tables(t, o, S, W) is None
+        acc = o if acc is None else oracle.merge(acc, o, S, W)
+    assert int(oracle.sections(acc, S, W)["counts"].sum()) > 0
+
+
+def test_reset_and_accumulate():
+    s, W, hdr, addr, val = random_trace(4242, n=4000)
+    d = to_device(s, hdr, addr, val)
+    ctx = sassi.Context(s, W, sassi.SASSI_H_ALL)
+    ctx.consume(d)
+    once = ctx.read_tables()
+    ctx.consume(d)
+    twice = ctx.read_tables()
+    o = oracle.run(s, W, oracle.H_ALL, hdr, addr, val)
+    oracle.consume(o, s, W, oracle.H_ALL, hdr, addr, val)
+    assert np.array_equal(twice, o)
+    ctx.reset()
+    ctx.consume(d)
+    assert np.array_equal(ctx.read_tables(), once)
+    with pytest.raises(sassi.SassiError):
+        sassi.sassi_attach_handler(ctx.handle, 1)    # after consume: ESTATE
+    ctx.close()
+
+
+def test_consume_host_equals_device():
+    P, mask, d = _gen("c2", limit=3_000_000)
+    h = gen.to_host(d)
+    t_dev = gpu_table(h["sites"], P.total_warps, mask, d)
+    ctx = sassi.Context(h["sites"], P.total_warps, mask)
+    hrec = dict(hdr=np.ascontiguousarray(h["hdr"]), addr=h["addr"], val=h["val"],
+                chunk_base=h["chunk_base"], n=h["n"], n_addr_rows=h["n_addr_rows"],
+                n_val_rows=h["n_val_rows"])
+    ctx.consume_host(hrec)
+    assert np.array_equal(ctx.read_tables(), t_dev)
+    ctx.close()
