@@ -55,8 +55,8 @@
  *   val[S][2]      warp executions, thread executions ("weight", Fig.9)
  *   ones[S][4]     constantOnes[d]  (low 32 bits used; init 0xFFFFFFFF)   (Fig.9)
  *   zeros[S][4]    constantZeros[d] (low 32 bits used; init 0xFFFFFFFF)   (Fig.9)
- *   nonscalar[S][4] warp executions whose lanes did not all write the same value to dst d;
- *                  the paper's isScalar[d] == (nonscalar[d] == 0)       (Fig.9)
+ *   scalar[S][4]   isScalar[d]: 1 iff in every warp execution all written lanes wrote one
+ *                  value to dst d (AND of allSame; init 1)            (Fig.9)
  *   h32[32][32]    sassi_counters[numActive-1][unique-1], unique = distinct 32 B sectors (Fig.6 l.33)
  *   h128[32][32]   the same matrix with 128 B lines
  *   counts[32*W]   per-thread eligible dynamic-instruction counts (§8.1 (4), L627)
@@ -159,7 +159,7 @@ typedef struct sassi_inj_site {
 } sassi_inj_site;      /* 32 B */
 
 typedef struct sassi_layout {
-  uint64_t diag, br, mem, val, ones, zeros, nonscalar, h32, h128, counts, total; /* in u64 words */
+  uint64_t diag, br, mem, val, ones, zeros, scalar, h32, h128, counts, total; /* in u64 words */
 } sassi_layout;
 
 /* Offsets of the table image (host-only arithmetic; no device needed). */

@@ -44,8 +44,8 @@ def layout(n_sites: int, n_warps: int) -> dict:
     L["val"] = L["mem"] + 4 * S
     L["ones"] = L["val"] + 2 * S
     L["zeros"] = L["ones"] + 4 * S
-    L["nonscalar"] = L["zeros"] + 4 * S
-    L["h32"] = L["nonscalar"] + 4 * S
+    L["scalar"] = L["zeros"] + 4 * S
+    L["h32"] = L["scalar"] + 4 * S
     L["h128"] = L["h32"] + 1024
     L["counts"] = L["h128"] + 1024
     L["total"] = L["counts"] + 32 * W
@@ -63,8 +63,8 @@ def sections(table: np.ndarray, n_sites: int, n_warps: int) -> dict:
         "mem": t[L["mem"]:L["val"]].reshape(S, 4),
         "val": t[L["val"]:L["ones"]].reshape(S, 2),
         "ones": t[L["ones"]:L["zeros"]].reshape(S, 4),
-        "zeros": t[L["zeros"]:L["nonscalar"]].reshape(S, 4),
-        "nonscalar": t[L["nonscalar"]:L["h32"]].reshape(S, 4),
+        "zeros": t[L["zeros"]:L["scalar"]].reshape(S, 4),
+        "scalar": t[L["scalar"]:L["h32"]].reshape(S, 4),
         "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
         "h128": t[L["h128"]:L["counts"]].reshape(32, 32),
         "counts": t[L["counts"]:L["total"]],

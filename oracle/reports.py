@@ -35,7 +35,7 @@ def value_profile_lines(table, sites, n_warps):
                     chars.append("0")
                 else:
                     chars.append("T")
-            star = "*" if int(sec["nonscalar"][s, d]) == 0 else ""
+            star = "*" if int(sec["scalar"][s, d]) == 1 else ""
             lines.append("R%d%s <- [%s]" % (int(site["reg_num"][d]), star, "".join(chars)))
         out.append((int(site["pc"]), lines))
     return out
@@ -77,7 +77,7 @@ def table2_percent(table, sites, n_warps):
         w = float(sec["val"][s, 1])
         for d in range(int(site["n_gpr_dst"])):
             const = bin((int(sec["ones"][s, d]) | int(sec["zeros"][s, d])) & 0xFFFFFFFF).count("1")
-            scalar = 1.0 if int(sec["nonscalar"][s, d]) == 0 else 0.0
+            scalar = 1.0 if int(sec["scalar"][s, d]) == 1 else 0.0
             cb_s += const / 32.0
             sc_s += scalar
             n_s += 1

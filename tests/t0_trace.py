@@ -100,7 +100,7 @@ EXPECT_H128 = {(31, 0): 2, (3, 0): 1, (30, 30): 1, (31, 1): 1}
 EXPECT_VAL = {1: [4, 100], 3: [2, 33], 4: [1, 32]}
 EXPECT_ONES = {1: 0x0, 3: 0x1, 4: 0x7}
 EXPECT_ZEROS = {1: 0xFFFFFFE0, 3: 0xFFFFFFFE, 4: 0xFFFFFFF8}
-EXPECT_NONSCALAR = {1: 2, 3: 0, 4: 0}
+EXPECT_SCALAR = {1: 0, 3: 1, 4: 1}
 
 
 def expect_counts():
@@ -134,10 +134,10 @@ def check_table(t, sec):
         assert list(map(int, sec["val"][s])) == EXPECT_VAL.get(s, [0, 0]), ("val", s)
         assert int(sec["ones"][s, 0]) == EXPECT_ONES.get(s, 0xFFFFFFFF), ("ones", s)
         assert int(sec["zeros"][s, 0]) == EXPECT_ZEROS.get(s, 0xFFFFFFFF), ("zeros", s)
-        assert int(sec["nonscalar"][s, 0]) == EXPECT_NONSCALAR.get(s, 0), ("nonscalar", s)
+        assert int(sec["scalar"][s, 0]) == EXPECT_SCALAR.get(s, 1), ("scalar", s)
         for d in range(1, 4):
             assert int(sec["ones"][s, d]) == 0xFFFFFFFF and int(sec["zeros"][s, d]) == 0xFFFFFFFF
-            assert int(sec["nonscalar"][s, d]) == 0
+            assert int(sec["scalar"][s, d]) == 1
     h32 = np.zeros((32, 32), np.uint64)
     for k, v in EXPECT_H32.items():
         h32[k] = v
