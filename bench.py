@@ -1,0 +1,361 @@
+#!/usr/bin/env python3
+"""bench.py — records/s and HBM GB/s of the SASSI handler fold on B200 (BASELINE.json metric).
+
+Workload (N=1): config c3 of BASELINE.json (the largest configuration that fits one GPU; c5, the
+8-GPU configuration, does not): an SGEMM/stencil-shaped trace of 10^8 warp-instruction records
+(~19 GB in HBM, >> the 126 MB L2, so no flush is needed between steps), all four handlers
+attached. One step = the whole hot path: sassi_reset (CUPTI launch-callback analogue) +
+sassi_consume (fused fold) + sassi_sample_sites (1,000 injection sites, L629) [+ sassi_merge over
+NCCL when N > 1]. Weak scaling: each rank folds its own 10^8-record shard (its own warp ids).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--workload c3|c2|c4]
+
+--impl reference times the oracle (plain single-threaded C++, oracle/) on the host cores on a
+bounded sample of the same workload — the only reference implementation this tier has.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "warp-instr records/sec & HBM GB/s (% peak) at 1/2/4/8 B200; instrumented slowdown"
+SPEC_HBM_GBS = 8000.0
+N_DRAWS = 1000
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c3", choices=["c2", "c3", "c4"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md, 6.65 TB/s)"
+
+
+def ncu_traffic(workload):
+    """dram read+write bytes per consume launch from the committed ncu --set full capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_consume_%s.json" % workload)
+    if os.path.exists(p):
+        try:
+            return float(json.load(open(p))["dram_bytes_per_launch"])
+        except Exception:
+            return None
+    return None
+
+
+class ClockSampler:
+    """Samples SM clock + throttle reasons with NVML during the timed region."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+    def __init__(self, index):
+        self.samples, self.reasons, self.stop_ev = [], 0, threading.Event()
+        self.max_mhz = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self.stop_ev.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            time.sleep(0.005)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop_ev.set()
+        if self.nv:
+            self.t.join()
+
+    def result(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["unavailable"]}
+        names = [n for b, n in self.REASONS.items() if self.reasons & b and n != "gpu_idle"]
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": names, "samples": len(self.samples)}
+
+
+def workload_program(name, world):
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
+    P, limit, _, desc = gen.preset(name)
+    P.total_warps = P.total_warps * world  # weak scaling: each rank owns one shard of warps
+    return P, limit, desc
+
+
+def algorithmic_bytes(rec, handlers):
+    """16 B per header + 256 B per addr row of a GLOBAL memory site (memdiv attached) + 128 B per
+    val row (value attached) — counted from the stream."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
+    sites = rec["sites"]
+    glob = [int(s["pc"]) for s in sites if (int(s["flags"]) & gen.F_MEM) and int(s["domain"]) == 0]
+    pcs = rec["hdr"][:, 0]
+    n_glob = int(torch.isin(pcs, torch.tensor(np.array(glob, np.int64).astype(np.int32),
+                                              device=pcs.device)).sum().item()) if glob else 0
+    b = 16 * rec["n"]
+    if handlers & 2:
+        b += 256 * n_glob
+    if handlers & 4:
+        b += 128 * rec["n_val_rows"]
+    return b, n_glob
+
+
+def run_reference(args, rank, world):
+    """Oracle on the host cores, on a bounded sample of the same workload (rank 0 only)."""
+    if rank != 0:
+        return
+    import oracle
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
+    P, limit, desc = workload_program(args.workload, 1)
+    mask = gen.PRESETS[args.workload][2]
+    sample_n = 1 << 21
+    rec = gen.generate_host(P, sample_n, 0, 1024)
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.run(rec["sites"], P.total_warps, mask, rec["hdr"], rec["addr"], rec["val"])
+        if i >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    tmax = max(sum(times), 1e-9)
+    v = args.steps * rec["n"] / tmax
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "records/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * tmax / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": args.workload + ": " + desc, "sample_records": rec["n"]},
+            "cpu_baseline": {"value": v, "unit": "records/s", "cores": 1, "kind": "oracle",
+                             "sample": "first %d records (warps 0..1023) of %s per step" %
+                                       (rec["n"], args.workload)},
+            "e2e": {"value": v, "unit": "records/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(args, d_rec, mask, P):
+    """The oracle as it stands, single-threaded, on a ~10-30 s bounded sample (rank 0, N=1)."""
+    import oracle
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
+    n = 1 << 22
+    pre_cb = d_rec["chunk_base"][n // 256].cpu().numpy().view(np.uint64)
+    pre = dict(d_rec, hdr=d_rec["hdr"][:n], addr=d_rec["addr"][: int(pre_cb[0])],
+               val=d_rec["val"][: int(pre_cb[1])], n=n, n_addr_rows=int(pre_cb[0]),
+               n_val_rows=int(pre_cb[1]))
+    h = gen.to_host(pre)
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"])
+        reps += 1
+        el = time.perf_counter() - t0
+        if el > 8.0 or reps >= 3:
+            break
+    return {"value": reps * n / el, "unit": "records/s", "cores": 1, "kind": "oracle",
+            "sample": "first %d records of the %s stream, %d repetition(s), %.1f s" %
+                      (n, args.workload, reps, el)}
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    P, limit, desc = workload_program(args.workload, world)
+    mask = gen.PRESETS[args.workload][2]
+    per = P.total_warps // world
+    rec = gen.generate_device(P, limit, rank * per, per, device=dev)
+    n = rec["n"]
+    alg_bytes, n_glob = algorithmic_bytes(rec, mask)
+    ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
+    comm = None
+    if world > 1:
+        uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if rank == 0:
+            uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
+        dist.broadcast(uid, 0)
+        comm = sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
+    stream = torch.cuda.current_stream(dev)
+    sample = bool(mask & 8)
+
+    def step(ev_c0=None, ev_c1=None):
+        ctx.reset(stream)
+        if ev_c0 is not None:
+            ev_c0.record(stream)
+        ctx.consume(rec, stream=stream)
+        if ev_c1 is not None:
+            ev_c1.record(stream)
+        if comm is not None:
+            ctx.merge(comm, stream)
+        if sample:
+            ctx.sample(N_DRAWS, 20150616, stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = ctx.kernel_launches()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        t_start.record(stream)
+        for k in range(args.steps):
+            step(*evs[k])
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches = ctx.kernel_launches() - launches0
+    ms = t_start.elapsed_time(t_end)
+    consume_ms = [a.elapsed_time(b) for a, b in evs]
+    if world > 1:
+        tt = torch.tensor([ms], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    sec = ms / 1e3
+    value = world * n * args.steps / sec
+    consume_avg_s = statistics.mean(consume_ms) / 1e3
+    peak, peak_src = measured_peaks()
+    achieved = alg_bytes / consume_avg_s / 1e9
+
+    # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e and rank == 0 and world == 1:
+        e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev)
+
+    cpu = None
+    if not args.no_cpu_baseline and rank == 0 and world == 1:
+        cpu = cpu_baseline(args, rec, mask, P)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": args.workload + ": " + desc + ", all four handlers + %d-site "
+                       "sampling" % N_DRAWS if sample else args.workload + ": " + desc,
+                       "records_per_gpu": n, "sites": len(rec["sites"]),
+                       "threads": 32 * P.total_warps, "handlers": mask,
+                       "stored_bytes_per_gpu": 16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"],
+                       "algorithmic_bytes_per_gpu": alg_bytes,
+                       "l2": "inputs (%.1f GB) exceed the 126 MB L2; no flush" % (
+                           (16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"]) / 1e9),
+                       "parallelism": "dp%d (warp-id shards, NCCL allreduce merge)" % world},
+            "hbm_gbs": world * alg_bytes * args.steps / sec / 1e9,
+            "hbm_frac_of_spec_8tbs": alg_bytes * args.steps / sec / 1e9 / SPEC_HBM_GBS,
+            "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
+                         "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "peak_source": peak_src,
+                         "traffic": ncu_traffic(args.workload),
+                         "algorithmic_bytes_per_launch": alg_bytes,
+                         "consume_ms_avg": consume_avg_s * 1e3,
+                         "consume_share_of_step": (consume_avg_s * 1e3) / (ms / args.steps)},
+            "gpu_launches": launches,
+            "clocks": clk.result(),
+        }
+        if e2e:
+            line["e2e"] = e2e
+        if cpu:
+            line["cpu_baseline"] = cpu
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        sassi.sassi_nccl_comm_destroy(comm)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def measure_e2e(rec, P, mask, n_e2e, dev):
+    """records/s through sassi_consume_host: pinned host buffers of the first n_e2e records, the
+    H2D copies (double-buffered inside the library) and the table read-back inside the timing."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    n_e2e = (n_e2e // 256) * 256
+    cb = rec["chunk_base"][: n_e2e // 256 + 1]
+    tail = cb[-1].cpu().numpy().view(np.uint64)
+    na, nv = int(tail[0]), int(tail[1])
+    h = dict(hdr=rec["hdr"][:n_e2e].cpu().pin_memory(), addr=rec["addr"][:na].cpu().pin_memory(),
+             val=rec["val"][:nv].cpu().pin_memory(), chunk_base=cb.cpu().pin_memory(), n=n_e2e,
+             n_addr_rows=na, n_val_rows=nv)
+    ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=dev.index)
+    stream = torch.cuda.current_stream(dev)
+    out = np.zeros(ctx.layout["total"], np.uint64)
+    for _ in range(2):
+        ctx.reset(stream)
+        ctx.consume_host(h, stream=stream)
+        sassi.sassi_read_tables(ctx.handle, out.size, stream, out)
+    reps = 3
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        ctx.reset(stream)
+        ctx.consume_host(h, stream=stream)
+        sassi.sassi_read_tables(ctx.handle, out.size, stream, out)
+    el = time.perf_counter() - t0
+    ctx.close()
+    h2d = 16 * n_e2e + 256 * na + 128 * nv + 16 * (n_e2e // 256 + 1)
+    return {"value": reps * n_e2e / el, "unit": "records/s", "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": 8 * ctx.layout["total"], "records_per_step": n_e2e,
+            "h2d_gbs": reps * h2d / el / 1e9,
+            "note": "pinned host buffers, first %d records; wall clock around consume_host + "
+                    "read_tables (which synchronise)" % n_e2e}
+
+
+if __name__ == "__main__":
+    main()

@@ -17,13 +17,14 @@ constexpr int kConsumeThreads = 256;          // 8 warps per CTA
 constexpr int kWarpsPerCta = kConsumeThreads / 32;
 constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 30;  // keeps every smem u32 partial < 2^32
 
-// Packed per-site info word in the hash (bit layout).
-constexpr uint32_t I_SITE_MASK = 0xFFFu;      // site index (registration order), < 4096
-constexpr uint32_t I_BRANCH = 1u << 12;       // COND_BRANCH site
-constexpr uint32_t I_ADDR_ROW = 1u << 13;     // record carries an addr row (MEM, any domain)
-constexpr uint32_t I_MEMDIV = 1u << 14;       // MEM && GLOBAL: folded by the memdiv handler
-constexpr uint32_t I_NDST_SHIFT = 15;         // 3 bits: n_gpr_dst
-constexpr uint32_t I_ELIGIBLE = 1u << 18;     // instcount-eligible (R12)
+// Packed per-site info word in the hash (bit layout). The companion cidx word holds the
+// site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).
+constexpr uint32_t I_BRANCH = 1u << 0;        // COND_BRANCH site
+constexpr uint32_t I_ADDR_ROW = 1u << 1;      // record carries an addr row (MEM, any domain)
+constexpr uint32_t I_MEMDIV = 1u << 2;        // MEM && GLOBAL: folded by the memdiv handler
+constexpr uint32_t I_ELIGIBLE = 1u << 3;      // instcount-eligible (R12)
+constexpr uint32_t I_NDST_SHIFT = 4;          // 3 bits: n_gpr_dst
+constexpr uint32_t I_VD0_SHIFT = 8;           // 16 bits: first value-destination state slot
 
 __host__ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
   h ^= h >> 16;
@@ -36,7 +37,7 @@ __host__ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
 
 // Table image offsets (u64 words), same formulas as sassi_table_layout().
 struct Offsets {
-  uint64_t br, mem, val, ones, zeros, nonscalar, h32, h128, counts, total;
+  uint64_t br, mem, val, ones, zeros, scalar, h32, h128, counts, total;
 };
 
 // Kernel parameter block of the fused consume kernel.
@@ -50,12 +51,13 @@ struct ConsumeParams {
   uint64_t arow_end, vrow_end;      // one past the last valid row index (bounds check)
   const uint32_t* hash;             // [3][cap]: keys, info, cidx
   uint32_t cap;                     // power of two
-  uint32_t nb, nm, nvw;             // smem counters: branch sites, memdiv sites, value words
+  uint32_t nb, nm, nv, nvd;         // branch sites, memdiv sites, value sites, value (site,dst)s
+  uint32_t pw;                      // private counter words per warp (16 B multiple)
+  uint32_t priv;                    // 1: per-warp private counters; 0: one shared set + atomics
   uint32_t n_warps;                 // per-thread count coverage (32 * n_warps threads)
-  uint32_t nv;                      // value sites (flush map entries)
   const uint32_t* flush_b;          // [nb] site index of branch compact slot
   const uint32_t* flush_m;          // [nm] site index of memdiv compact slot
-  const uint32_t* flush_v;          // [nv][3] site index, word offset, n_dst
+  const uint32_t* flush_v;          // [nv][3] site index, first value-dst slot, n_dst
   uint64_t* table;                  // device table image
   Offsets off;
   uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
@@ -75,7 +77,7 @@ struct sassi_ctx {
   uint64_t* d_table = nullptr;
   uint32_t* d_hash = nullptr;       // [3][cap]
   uint32_t cap = 0;
-  uint32_t nb = 0, nm = 0, nv = 0, nvw = 0;
+  uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
   uint32_t* d_err = nullptr;
   uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums

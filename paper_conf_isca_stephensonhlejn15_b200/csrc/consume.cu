@@ -29,12 +29,6 @@ __device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t* p) {
   asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(r) : "l"(p));
   return r;
 }
-__device__ __forceinline__ uint32_t ld_nc_u32(const uint32_t* p) {
-  uint32_t r;
-  asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
-  return r;
-}
-
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src);
   uint32_t hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src);
@@ -92,6 +86,49 @@ __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane
   }
 }
 
+// Per-record counter update into the warp's private counter words: lanes whose records hit the
+// same site in this batch (short loop bodies) are detected with MATCH.ANY and fall back to
+// shared-memory atomics; all other lanes do a plain vector read-modify-write.
+__device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, uint32_t* region,
+                                              uint32_t priv, uint32_t lane) {
+  const uint32_t part = __ballot_sync(FULL, pred);
+  if (part == 0) return;
+  bool dup = !priv;
+  if (priv && pred) dup = __match_any_sync(part, off) != (1u << lane);
+  if (pred && !dup) {
+    uint4* q = reinterpret_cast<uint4*>(region + off);
+    uint4 c = *q;
+    c.x += v.x;
+    c.y += v.y;
+    c.z += v.z;
+    c.w += v.w;
+    *q = c;
+  } else if (pred) {
+    atomicAdd(region + off, v.x);
+    atomicAdd(region + off + 1, v.y);
+    atomicAdd(region + off + 2, v.z);
+    if (v.w) atomicAdd(region + off + 3, v.w);
+  }
+}
+
+__device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, uint32_t* region,
+                                              uint32_t priv, uint32_t lane) {
+  const uint32_t part = __ballot_sync(FULL, pred);
+  if (part == 0) return;
+  bool dup = !priv;
+  if (priv && pred) dup = __match_any_sync(part, off) != (1u << lane);
+  if (pred && !dup) {
+    uint2* q = reinterpret_cast<uint2*>(region + off);
+    uint2 c = *q;
+    c.x += v.x;
+    c.y += v.y;
+    *q = c;
+  } else if (pred) {
+    atomicAdd(region + off, v.x);
+    atomicAdd(region + off + 1, v.y);
+  }
+}
+
 template <uint32_t H>
 __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(16) uint32_t sm[];
@@ -99,14 +136,15 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   uint32_t* s_keys = sm;
   uint32_t* s_info = sm + cap;
   uint32_t* s_cidx = sm + 2 * cap;
-  uint32_t* s_br = sm + 3 * cap;        // [nb][4]: total, active, taken, divergent
-  uint32_t* s_mem = s_br + 4 * p.nb;    // [nm][4]: warps, lanes, sectors, lines
-  uint32_t* s_val = s_mem + 4 * p.nm;   // per value site: we, te, {ones, zeros, nonscalar} x ndst
-  uint32_t* s_h32 = s_val + p.nvw;      // [32][32]
-  uint32_t* s_h128 = s_h32 + 1024;      // [32][32]
-  uint32_t* s_diag = s_h128 + 1024;     // n_records, n_invalid, n_unknown, n_bad_warp (+pad)
-  const uint32_t desc_word = (3 * cap + 4 * (p.nb + p.nm) + p.nvw + 2048 + 8 + 1) & ~1u;
-  uint2* s_vdesc = reinterpret_cast<uint2*>(sm + desc_word);  // [warps][128] value-row descriptors
+  uint32_t o = (3 * cap + 3) & ~3u;
+  uint4* s_vstate = reinterpret_cast<uint4*>(sm + o);  // [nvd]: ones, zeros, isScalar, -
+  o += 4 * p.nvd;
+  uint32_t* s_h32 = sm + o;                             // [32][32]
+  uint32_t* s_h128 = s_h32 + 1024;                      // [32][32]
+  uint32_t* s_diag = s_h128 + 1024;                     // 8 words
+  uint32_t* s_priv = s_diag + 8;                        // [warps or 1][pw] counters
+  const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
+  uint2* s_vdesc = reinterpret_cast<uint2*>(s_priv + n_regions * p.pw);  // [warps][128]
 
   const uint32_t tid = threadIdx.x;
   for (uint32_t i = tid; i < cap; i += blockDim.x) {
@@ -114,22 +152,15 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
     s_info[i] = p.hash[cap + i];
     s_cidx[i] = p.hash[2 * cap + i];
   }
-  for (uint32_t i = tid; i < 4 * (p.nb + p.nm) + p.nvw + 2048 + 8; i += blockDim.x) s_br[i] = 0;
-  __syncthreads();
-  if (H & SASSI_H_VALUE) {
-    for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
-      const uint32_t off = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
-      for (uint32_t d = 0; d < nd; ++d) {
-        s_val[off + 2 + 3 * d] = FULL;  // constantOnes: AND identity
-        s_val[off + 3 + 3 * d] = FULL;  // constantZeros
-      }
-    }
-  }
+  for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
+  for (uint32_t i = tid; i < 2048 + 8 + n_regions * p.pw; i += blockDim.x) s_h32[i] = 0;
   __syncthreads();
 
   const uint32_t lane = tid & 31u, wib = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
+  uint32_t* wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
   uint2* vdesc = s_vdesc + wib * 128;
+  const uint32_t PB = 4 * p.nb, PV = 4 * p.nb + 4 * p.nm;
   const uint64_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta;
   uint32_t c_rec = 0, c_inv = 0, c_unk = 0, c_bad = 0;
@@ -140,12 +171,18 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   for (uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
     const ulonglong2 cb0 = p.cb[u];
     const ulonglong2 cb1 = p.cb[u + 1];
+    if (!(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end && cb0.y >= p.vrow_base &&
+          cb0.y <= cb1.y && cb1.y <= p.vrow_end)) {
+      err |= 8u;  // chunk index outside the row buffers
+      continue;
+    }
     uint64_t arow = cb0.x, vrow = cb0.y;
     const uint64_t rec0 = u * SASSI_CHUNK;
     const uint64_t left = p.n - rec0;
     const uint32_t nbat = left >= SASSI_CHUNK ? SASSI_CHUNK / 32 : (uint32_t)((left + 31) / 32);
     uint4 hnext = (rec0 + lane < p.n) ? ld_nc_v4(p.hdr + rec0 + lane) : make_uint4(EMPTY_KEY, 0, 0, 0);
-    for (uint32_t b = 0; b < nbat; ++b) {
+    uint32_t b = 0;
+    for (; b < nbat; ++b) {
       const uint64_t i = rec0 + 32 * b + lane;
       const bool valid = i < p.n;
       const uint4 h = hnext;
@@ -173,11 +210,8 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       c_rec += valid;
       c_unk += valid && !known;
       // ---- row indices of this batch (rows follow their records) ----
-      const bool has_a = known && (info & I_ADDR_ROW);
+      const uint32_t ma = __ballot_sync(FULL, known && (info & I_ADDR_ROW));
       const uint32_t nd = known ? (info >> I_NDST_SHIFT) & 7u : 0u;
-      const uint32_t ma = __ballot_sync(FULL, has_a);
-      const uint64_t my_arow = arow + __popc(ma & lt);
-      arow += __popc(ma);
       uint32_t vpre = 0, vtot = 0;
 #pragma unroll
       for (int k = 0; k < 3; ++k) {
@@ -185,8 +219,13 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
         vpre += __popc(mk & lt) << k;
         vtot += __popc(mk) << k;
       }
-      const uint64_t bv0 = vrow;
+      const uint64_t arow_b = arow, vrow_b = vrow;
+      arow += __popc(ma);
       vrow += vtot;
+      if (arow > cb1.x || vrow > cb1.y) {
+        err |= 4u;  // rows of this batch run past the chunk's rows: stream inconsistent
+        break;
+      }
       const uint32_t act = h.z, m2 = h.w;
       const bool live = known && act != 0;
       c_inv += known && act == 0;
@@ -194,14 +233,11 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
 
       // ---- Case study I: branch divergence (Fig.4) ----
       if (H & SASSI_H_BRANCH) {
-        if (live && (info & I_BRANCH)) {
-          uint32_t* st = s_br + 4 * (cidx & 0xFFFFu);
-          const uint32_t T = G;  // taken = mask2 & active (R1)
-          atomicAdd(st + 0, 1u);
-          atomicAdd(st + 1, (uint32_t)__popc(act));
-          atomicAdd(st + 2, (uint32_t)__popc(T));
-          if (T != 0 && T != act) atomicAdd(st + 3, 1u);
-        }
+        const bool isb = live && (info & I_BRANCH);
+        add_counters4(isb, 4 * (cidx & 0xFFFFu),
+                      make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
+                                 (G != 0 && G != act) ? 1u : 0u),
+                      wpriv, p.priv, lane);
       }
       // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
       if (H & SASSI_H_INSTCOUNT) {
@@ -216,7 +252,8 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
           const bool mine = E != 0 && h.y == w0;
           const uint32_t cnt = __popc(transpose32(mine ? E : 0u, lane));
           if (w0 != acc_w) {
-            if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+            if (acc_w != FULL && acc)
+              atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
             acc_w = w0;
             acc = 0;
           }
@@ -225,9 +262,11 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
           if (mine) E = 0;
         }
       }
-      // ---- Case study II: memory address divergence (Fig.6) ----
+      // ---- Case study II: memory address divergence (Fig.6), one warp per address row ----
       if (H & SASSI_H_MEMDIV) {
         uint32_t selm = __ballot_sync(FULL, live && (info & I_MEMDIV) && G != 0);
+        const uint64_t* abase = p.addr + 32ull * (arow_b - p.arow_base) + lane;
+        const uint32_t arel = __popc(ma & lt);
         while (selm) {
           uint64_t a[4];
           uint32_t g[4], mi[4];
@@ -237,15 +276,10 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
             if (selm) {
               const int j = __ffs(selm) - 1;
               selm &= selm - 1;
-              const uint64_t row = shfl64(my_arow, j);
+              const uint32_t r = __shfl_sync(FULL, arel, j);
               g[k] = __shfl_sync(FULL, G, j);
               mi[k] = __shfl_sync(FULL, cidx & 0xFFFFu, j);
-              if (row < p.arow_base || row >= p.arow_end) {
-                err |= 1u;
-                g[k] = 0;
-              } else {
-                a[k] = ld_nc_u64(p.addr + 32ull * (row - p.arow_base) + lane);
-              }
+              a[k] = ld_nc_u64(abase + 32 * r);
             }
           }
 #pragma unroll
@@ -254,64 +288,73 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
               uint32_t s, L;
               memdiv_row(a[k], g[k], lane, &s, &L);
               const uint32_t n = __popc(g[k]);
-              if (lane < 6) {
-                uint32_t* dst;
-                uint32_t v = 1;
-                if (lane == 0) dst = s_h32 + 32 * (n - 1) + (s - 1);
-                else if (lane == 1) dst = s_h128 + 32 * (n - 1) + (L - 1);
-                else {
-                  dst = s_mem + 4 * mi[k] + (lane - 2);
-                  v = lane == 2 ? 1u : (lane == 3 ? n : (lane == 4 ? s : L));
+              if (lane < 2)
+                atomicAdd(lane == 0 ? s_h32 + 32 * (n - 1) + (s - 1) : s_h128 + 32 * (n - 1) + (L - 1), 1u);
+              uint32_t* q = wpriv + PB + 4 * mi[k];
+              if (p.priv) {
+                if (lane == 0) {
+                  uint4 c = *reinterpret_cast<uint4*>(q);
+                  c.x += 1;
+                  c.y += n;
+                  c.z += s;
+                  c.w += L;
+                  *reinterpret_cast<uint4*>(q) = c;
                 }
-                atomicAdd(dst, v);
+              } else if (lane >= 2 && lane < 6) {
+                atomicAdd(q + (lane - 2), lane == 2 ? 1u : (lane == 3 ? n : (lane == 4 ? s : L)));
               }
             }
           }
         }
       }
-      // ---- Case study III: value profiling (Fig.9) ----
+      // ---- Case study III: value profiling (Fig.9), 4 value rows per 128-bit warp load ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
-        const uint32_t voff = cidx >> 16;
-        if (selv) {
-          atomicAdd(s_val + voff, 1u);                       // warp executions
-          atomicAdd(s_val + voff + 1, (uint32_t)__popc(G));  // thread executions ("weight")
-        }
-        for (uint32_t d = 0; d < nd; ++d) vdesc[vpre + d] = make_uint2(selv ? G : 0u, voff + 2 + 3 * d);
+        add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
+                      p.priv, lane);
+        const uint32_t vd0 = info >> I_VD0_SHIFT;
+        for (uint32_t d = 0; d < nd; ++d) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
         __syncwarp();
-        for (uint32_t r0 = 0; r0 < vtot; r0 += 8) {
-          uint32_t v[8];
-          uint2 dsc[8];
+        // quad q = rows 4q..4q+3 of this batch; lane holds row 4q + lane/8, columns 4*(lane%8)..+3
+        const uint4* vq = reinterpret_cast<const uint4*>(p.val + 32ull * (vrow_b - p.vrow_base)) + lane;
+        const uint32_t nq = (vtot + 3) >> 2;
+        const uint32_t sh = (lane & 7u) * 4;
+        for (uint32_t q0 = 0; q0 < nq; q0 += 4) {
+          uint4 x[4];
 #pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            const uint32_t r = r0 + k;
-            dsc[k] = r < vtot ? vdesc[r] : make_uint2(0u, 0u);
-            if (dsc[k].x) {
-              const uint64_t row = bv0 + r;
-              if (row < p.vrow_base || row >= p.vrow_end) {
-                err |= 2u;
-                dsc[k].x = 0;
-              } else {
-                v[k] = ld_nc_u32(p.val + 32ull * (row - p.vrow_base) + lane);
-              }
-            }
+          for (int k = 0; k < 4; ++k) {
+            const uint32_t rr = 4 * (q0 + k) + (lane >> 3);
+            x[k] = rr < vtot ? ld_nc_v4(vq + 32 * (q0 + k)) : make_uint4(0, 0, 0, 0);
           }
 #pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            if (dsc[k].x) {
-              const uint32_t V = dsc[k].x;
-              const bool in = (V >> lane) & 1u;
-              const uint32_t va = __reduce_and_sync(FULL, in ? v[k] : FULL);
-              const uint32_t vo = __reduce_or_sync(FULL, in ? v[k] : 0u);
-              uint32_t* w = s_val + dsc[k].y;
-              if (lane == 0) {
-                const uint32_t cur = w[0];
-                if ((cur & va) != cur) atomicAnd(w + 0, va);         // atomicAnd(constantOnes, v)
-              } else if (lane == 1) {
-                const uint32_t cur = w[1];
-                if ((cur & ~vo) != cur) atomicAnd(w + 1, ~vo);       // atomicAnd(constantZeros, ~v)
-              } else if (lane == 2) {
-                if (va != vo) atomicAdd(w + 2, 1u);                  // not all lanes equal
+          for (int k = 0; k < 4; ++k) {
+            if (q0 + k < nq) {
+              const uint32_t rr = 4 * (q0 + k) + (lane >> 3);
+              const uint2 ds = rr < vtot ? vdesc[rr] : make_uint2(0u, 0u);
+              const uint32_t vb = (ds.x >> sh) & 0xFu;
+              uint32_t va, vo;
+              if (__all_sync(FULL, vb == 0xFu || ds.x == 0)) {
+                va = x[k].x & x[k].y & x[k].z & x[k].w;
+                vo = x[k].x | x[k].y | x[k].z | x[k].w;
+              } else {
+                const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
+                const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - (vb >> 3);
+                va = (x[k].x | ~m0) & (x[k].y | ~m1) & (x[k].z | ~m2_) & (x[k].w | ~m3);
+                vo = (x[k].x & m0) | (x[k].y & m1) | (x[k].z & m2_) | (x[k].w & m3);
+              }
+              va &= __shfl_xor_sync(FULL, va, 1);
+              vo |= __shfl_xor_sync(FULL, vo, 1);
+              va &= __shfl_xor_sync(FULL, va, 2);
+              vo |= __shfl_xor_sync(FULL, vo, 2);
+              va &= __shfl_xor_sync(FULL, va, 4);
+              vo |= __shfl_xor_sync(FULL, vo, 4);
+              if ((lane & 7u) == 0 && ds.x != 0) {
+                uint4* st = s_vstate + ds.y;
+                const uint4 c = *st;
+                const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
+                if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
+                if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
+                if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
               }
             }
           }
@@ -319,7 +362,7 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
         __syncwarp();
       }
     }
-    if (lane == 0 && (arow != cb1.x || vrow != cb1.y)) err |= 4u;  // chunk index inconsistent
+    if (b == nbat && lane == 0 && (arow != cb1.x || vrow != cb1.y)) err |= 4u;  // index disagrees
   }
   if (H & SASSI_H_INSTCOUNT) {
     if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
@@ -339,26 +382,40 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   }
   __syncthreads();
 
-  // ---- flush the CTA's shared-memory partials into the global u64 image ----
+  // ---- flush: sum the warps' private counters, fold into the global u64 image ----
   if (tid < 4 && s_diag[tid]) atomicAdd(&table[tid], (unsigned long long)s_diag[tid]);
+  auto sum_words = [&](uint32_t off) -> uint4 {
+    uint4 t = make_uint4(0, 0, 0, 0);
+    for (uint32_t w = 0; w < n_regions; ++w) {
+      const uint32_t* q = s_priv + w * p.pw + off;
+      t.x += q[0];
+      t.y += q[1];
+      t.z += q[2];
+      t.w += q[3];
+    }
+    return t;
+  };
   if (H & SASSI_H_BRANCH) {
-    for (uint32_t b = tid; b < p.nb; b += blockDim.x) {
-      const uint32_t* st = s_br + 4 * b;
-      if (st[0] == 0) continue;
-      unsigned long long* g = table + p.off.br + 5ull * p.flush_b[b];
-      atomicAdd(g + 0, (unsigned long long)st[0]);
-      atomicAdd(g + 1, (unsigned long long)st[1]);
-      if (st[2]) atomicAdd(g + 2, (unsigned long long)st[2]);
-      if (st[1] - st[2]) atomicAdd(g + 3, (unsigned long long)(st[1] - st[2]));  // not taken
-      if (st[3]) atomicAdd(g + 4, (unsigned long long)st[3]);
+    for (uint32_t bi = tid; bi < p.nb; bi += blockDim.x) {
+      const uint4 t = sum_words(4 * bi);
+      if (t.x == 0) continue;
+      unsigned long long* g = table + p.off.br + 5ull * p.flush_b[bi];
+      atomicAdd(g + 0, (unsigned long long)t.x);
+      atomicAdd(g + 1, (unsigned long long)t.y);
+      if (t.z) atomicAdd(g + 2, (unsigned long long)t.z);
+      if (t.y - t.z) atomicAdd(g + 3, (unsigned long long)(t.y - t.z));  // not taken = active - taken
+      if (t.w) atomicAdd(g + 4, (unsigned long long)t.w);
     }
   }
   if (H & SASSI_H_MEMDIV) {
     for (uint32_t m = tid; m < p.nm; m += blockDim.x) {
-      const uint32_t* st = s_mem + 4 * m;
-      if (st[0] == 0) continue;
+      const uint4 t = sum_words(PB + 4 * m);
+      if (t.x == 0) continue;
       unsigned long long* g = table + p.off.mem + 4ull * p.flush_m[m];
-      for (int f = 0; f < 4; ++f) atomicAdd(g + f, (unsigned long long)st[f]);
+      atomicAdd(g + 0, (unsigned long long)t.x);
+      atomicAdd(g + 1, (unsigned long long)t.y);
+      atomicAdd(g + 2, (unsigned long long)t.z);
+      atomicAdd(g + 3, (unsigned long long)t.w);
     }
     for (uint32_t c = tid; c < 2048; c += blockDim.x) {
       const uint32_t v = s_h32[c];
@@ -367,16 +424,20 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   }
   if (H & SASSI_H_VALUE) {
     for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
-      const uint32_t site = p.flush_v[3 * k], off = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
-      const uint32_t* w = s_val + off;
-      if (w[0] == 0) continue;
-      atomicAdd(table + p.off.val + 2ull * site, (unsigned long long)w[0]);
-      atomicAdd(table + p.off.val + 2ull * site + 1, (unsigned long long)w[1]);
+      const uint32_t site = p.flush_v[3 * k], vd0 = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
+      uint32_t we = 0, te = 0;
+      for (uint32_t w = 0; w < n_regions; ++w) {
+        we += s_priv[w * p.pw + PV + 2 * k];
+        te += s_priv[w * p.pw + PV + 2 * k + 1];
+      }
+      if (we == 0) continue;
+      atomicAdd(table + p.off.val + 2ull * site, (unsigned long long)we);
+      atomicAdd(table + p.off.val + 2ull * site + 1, (unsigned long long)te);
       for (uint32_t d = 0; d < nd; ++d) {
-        const uint32_t o = w[2 + 3 * d], z = w[3 + 3 * d], ns = w[4 + 3 * d];
-        if (o != FULL) atomicAnd(table + p.off.ones + 4ull * site + d, (unsigned long long)o);
-        if (z != FULL) atomicAnd(table + p.off.zeros + 4ull * site + d, (unsigned long long)z);
-        if (ns) atomicAdd(table + p.off.nonscalar + 4ull * site + d, (unsigned long long)ns);
+        const uint4 st = s_vstate[vd0 + d];
+        if (st.x != FULL) atomicAnd(table + p.off.ones + 4ull * site + d, (unsigned long long)st.x);
+        if (st.y != FULL) atomicAnd(table + p.off.zeros + 4ull * site + d, (unsigned long long)st.y);
+        if (st.z != 1u) atomicAnd(table + p.off.scalar + 4ull * site + d, 0ull);
       }
     }
   }
@@ -413,7 +474,8 @@ KernelFn select_kernel(uint32_t mask) {
 }  // namespace
 
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
-  size_t words = 3ull * c->cap + 4ull * (c->nb + c->nm) + c->nvw + 2048 + 8;
+  size_t words = (3ull * c->cap + 3) & ~3ull;
+  words += 4ull * c->nvd + 2048 + 8 + (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
   words = (words + 1) & ~1ull;  // 8-byte align the descriptor area
   *bytes = 4 * words + sizeof(uint2) * 128 * kWarpsPerCta;
   return 0;

@@ -70,28 +70,33 @@ int nccl_err(ncclResult_t r, const char* what) {
   return set_error(SASSI_ENCCL, std::string(what) + ": " + nccl().GetErrorString(r));
 }
 
-// packed image: [4 diag sums][br..val sums][nonscalar..counts sums][8S masks x 4 words]
+// packed image: [4 diag][br..val sums][h32..counts sums][isScalar 0/1 sums, 4S][ones+zeros masks
+// byte-expanded, 8S x 4 words]. After the sum: isScalar = (sum == nranks); mask bit set iff its
+// byte == nranks.
 struct PackLayout {
-  uint64_t n_sum_a, n_sum_b, n_mask_words, total;
+  uint64_t n_sum_a, n_sum_b, n_scalar, n_mask_words, total;
 };
 PackLayout pack_layout(const sassi_ctx* c) {
   PackLayout L;
   L.n_sum_a = c->off.ones - c->off.br;
-  L.n_sum_b = c->off.total - c->off.nonscalar;
+  L.n_sum_b = c->off.total - c->off.h32;
+  L.n_scalar = 4ull * c->S;
   L.n_mask_words = 8ull * c->S * 4;
-  L.total = 4 + L.n_sum_a + L.n_sum_b + L.n_mask_words;
+  L.total = 4 + L.n_sum_a + L.n_sum_b + L.n_scalar + L.n_mask_words;
   return L;
 }
 
 __global__ void pack_kernel(const uint64_t* __restrict__ t, Offsets o, PackLayout L, uint64_t* pk) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t b1 = 4 + L.n_sum_a, b2 = b1 + L.n_sum_b, b3 = b2 + L.n_scalar;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < L.total; i += stride) {
     uint64_t v;
     if (i < 4) v = t[i];
-    else if (i < 4 + L.n_sum_a) v = t[o.br + (i - 4)];
-    else if (i < 4 + L.n_sum_a + L.n_sum_b) v = t[o.nonscalar + (i - 4 - L.n_sum_a)];
+    else if (i < b1) v = t[o.br + (i - 4)];
+    else if (i < b2) v = t[o.h32 + (i - b1)];
+    else if (i < b3) v = t[o.scalar + (i - b2)];
     else {
-      const uint64_t w = i - (4 + L.n_sum_a + L.n_sum_b);
+      const uint64_t w = i - b3;
       const uint32_t mask = (uint32_t)t[o.ones + w / 4];  // ones[S][4] then zeros[S][4]
       const uint32_t byte8 = (mask >> (8 * (w % 4))) & 0xFFu;
       v = 0;
@@ -104,16 +109,17 @@ __global__ void pack_kernel(const uint64_t* __restrict__ t, Offsets o, PackLayou
 
 __global__ void unpack_kernel(uint64_t* __restrict__ t, Offsets o, PackLayout L,
                               const uint64_t* __restrict__ pk, uint32_t nranks) {
-  const uint64_t n_masks = L.n_mask_words / 4;
-  const uint64_t n_items = 4 + L.n_sum_a + L.n_sum_b + n_masks;
+  const uint64_t b1 = 4 + L.n_sum_a, b2 = b1 + L.n_sum_b, b3 = b2 + L.n_scalar;
+  const uint64_t n_items = b3 + L.n_mask_words / 4;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_items; i += stride) {
     if (i < 4) t[i] = pk[i];
-    else if (i < 4 + L.n_sum_a) t[o.br + (i - 4)] = pk[i];
-    else if (i < 4 + L.n_sum_a + L.n_sum_b) t[o.nonscalar + (i - 4 - L.n_sum_a)] = pk[i];
+    else if (i < b1) t[o.br + (i - 4)] = pk[i];
+    else if (i < b2) t[o.h32 + (i - b1)] = pk[i];
+    else if (i < b3) t[o.scalar + (i - b2)] = pk[i] == nranks ? 1ull : 0ull;
     else {
-      const uint64_t m = i - (4 + L.n_sum_a + L.n_sum_b);
-      const uint64_t* w = pk + 4 + L.n_sum_a + L.n_sum_b + 4 * m;
+      const uint64_t m = i - b3;
+      const uint64_t* w = pk + b3 + 4 * m;
       uint32_t mask = 0;
       for (int q = 0; q < 4; ++q)
         for (int b = 0; b < 8; ++b)

@@ -10,8 +10,8 @@ Offsets layout_offsets(uint32_t S, uint32_t W) {
   o.val = o.mem + 4ull * S;
   o.ones = o.val + 2ull * S;
   o.zeros = o.ones + 4ull * S;
-  o.nonscalar = o.zeros + 4ull * S;
-  o.h32 = o.nonscalar + 4ull * S;
+  o.scalar = o.zeros + 4ull * S;
+  o.h32 = o.scalar + 4ull * S;
   o.h128 = o.h32 + 1024;
   o.counts = o.h128 + 1024;
   o.total = o.counts + 32ull * W;
@@ -20,13 +20,15 @@ Offsets layout_offsets(uint32_t S, uint32_t W) {
 
 namespace {
 
-// Sums start at 0; constantOnes / constantZeros start all-ones (the AND identity, Fig.9);
+// Sums start at 0; constantOnes / constantZeros start all-ones and isScalar starts 1 (the AND
+// identities, Fig.9);
 // diag[4..7] describe the image.
 __global__ void init_tables_kernel(uint64_t* t, Offsets o, uint32_t S, uint32_t W, uint32_t mask) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < o.total; i += stride) {
     uint64_t v = 0;
-    if (i >= o.ones && i < o.nonscalar) v = 0xFFFFFFFFull;
+    if (i >= o.ones && i < o.scalar) v = 0xFFFFFFFFull;
+    else if (i >= o.scalar && i < o.h32) v = 1;
     else if (i == 4) v = S;
     else if (i == 5) v = W;
     else if (i == 6) v = mask;
@@ -57,7 +59,7 @@ extern "C" int sassi_table_layout(uint32_t n_sites, uint32_t n_warps, sassi_layo
   out->val = o.val;
   out->ones = o.ones;
   out->zeros = o.zeros;
-  out->nonscalar = o.nonscalar;
+  out->scalar = o.scalar;
   out->h32 = o.h32;
   out->h128 = o.h128;
   out->counts = o.counts;

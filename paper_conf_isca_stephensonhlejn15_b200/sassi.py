@@ -35,7 +35,7 @@ class SassiRecords(ctypes.Structure):
 
 
 class SassiLayout(ctypes.Structure):
-    _fields_ = [(k, _u64) for k in ("diag", "br", "mem", "val", "ones", "zeros", "nonscalar", "h32",
+    _fields_ = [(k, _u64) for k in ("diag", "br", "mem", "val", "ones", "zeros", "scalar", "h32",
                                     "h128", "counts", "total")]
 
 
@@ -247,8 +247,8 @@ class Context:
         return {"diag": t[0:8], "br": t[L["br"]:L["mem"]].reshape(S, 5),
                 "mem": t[L["mem"]:L["val"]].reshape(S, 4), "val": t[L["val"]:L["ones"]].reshape(S, 2),
                 "ones": t[L["ones"]:L["zeros"]].reshape(S, 4),
-                "zeros": t[L["zeros"]:L["nonscalar"]].reshape(S, 4),
-                "nonscalar": t[L["nonscalar"]:L["h32"]].reshape(S, 4),
+                "zeros": t[L["zeros"]:L["scalar"]].reshape(S, 4),
+                "scalar": t[L["scalar"]:L["h32"]].reshape(S, 4),
                 "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
                 "h128": t[L["h128"]:L["counts"]].reshape(32, 32), "counts": t[L["counts"]:L["total"]]}
 
