@@ -6,8 +6,10 @@
 //   branch     Fig.4 (L237-L243)   lane-per-record: popc of active / taken masks
 //   memdiv     Fig.6 (L361-L369)   warp-per-row: distinct 32 B sectors and 128 B lines among the
 //                                  guard-true lanes; window-bitmap REDUX fast path, MATCH.ANY slow path
-//   value      Fig.9 (L549-L563)   warp-per-row: REDUX.AND / REDUX.OR over written lanes ->
-//                                  constant ones / zeros and "all lanes same" (scalar)
+//   value      Fig.9 (L549-L563)   row-per-lane: a batch's contiguous value rows are bulk-copied
+//                                  (TMA, cp.async.bulk + mbarrier) into the warp's shared-memory
+//                                  buffer; lane j folds row j's 32 values (AND / OR of the written
+//                                  lanes) -> constantOnes / constantZeros / isScalar
 //   instcount  §8.1 (L625-L627)    lane-per-record: 32x32 bit-matrix transpose + popc gives the
 //                                  per-lane count of 32 records; register accumulator per trace warp
 // Work split: a warp owns one 256-record chunk at a time (chunk_base gives its row offsets) and walks
@@ -29,12 +31,6 @@ __device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t* p) {
   asm volatile("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(r) : "l"(p));
   return r;
 }
-__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
-  uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src);
-  uint32_t hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src);
-  return ((uint64_t)hi << 32) | lo;
-}
-
 // 32x32 bit-matrix transpose across the warp: in, lane i holds row i; out, lane l holds the word
 // whose bit i is bit l of row i. Five butterfly stages swapping off-diagonal blocks.
 __device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
@@ -55,24 +51,23 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
 }
 
 // Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
-// over the lanes of G. Fast path when every sector lies within [-32, 31] of the first lane's: a
-// 64-bit window bitmap OR-reduced across the warp. Otherwise MATCH.ANY groups equal keys.
+// over the lanes of G. Fast path when every sector lies within [-32, 31] of the first G lane's (same
+// high word): a 64-bit window bitmap OR-reduced across the warp (REDUX). Otherwise MATCH.ANY groups
+// equal keys and the group leaders are counted.
 __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
                                            uint32_t* out_l) {
   const bool in = (G >> lane) & 1u;
   const uint64_t sec = a >> 5;
+  const uint32_t slo = (uint32_t)sec, shi = (uint32_t)(sec >> 32);
   const int leader = __ffs(G) - 1;
-  const uint64_t base = shfl64(sec, leader);
-  const int64_t d = (int64_t)(sec - base);
-  const bool inwin = (uint64_t)(d + 32) < 64ull;
-  if (__all_sync(FULL, !in || inwin)) {
-    const uint64_t bit = in ? (1ull << (d + 32)) : 0ull;
-    const uint32_t lo = __reduce_or_sync(FULL, (uint32_t)bit);
-    const uint32_t hi = __reduce_or_sync(FULL, (uint32_t)(bit >> 32));
-    const int64_t dl = (int64_t)((sec >> 2) - (base >> 2));  // in [-8, 8]
-    const uint32_t lb = in ? (1u << (uint32_t)(dl + 8)) : 0u;
+  const uint32_t blo = __shfl_sync(FULL, slo, leader), bhi = __shfl_sync(FULL, shi, leader);
+  const uint32_t e = slo - blo + 32u;  // window position, valid when < 64 and high words agree
+  if (__all_sync(FULL, !in || (e < 64u && shi == bhi))) {
+    const uint32_t lo = __reduce_or_sync(FULL, in ? (1u << e) : 0u);          // e >= 32 -> 0
+    const uint32_t hi = __reduce_or_sync(FULL, in ? (1u << (e - 32u)) : 0u);  // e < 32 -> 0
+    const uint32_t ln = (uint32_t)(((int32_t)(e - 32u) + (int32_t)(blo & 3u)) >> 2) + 8u;  // 0..16
     *out_s = __popc(lo) + __popc(hi);
-    *out_l = __popc(__reduce_or_sync(FULL, lb));
+    *out_l = __popc(__reduce_or_sync(FULL, in ? (1u << ln) : 0u));
   } else {
     uint32_t gs = 0, gl = 0;
     if (in) {
@@ -83,6 +78,37 @@ __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane
     const bool ll = in && (uint32_t)(__ffs(gl) - 1) == lane;
     *out_s = __popc(__ballot_sync(FULL, ls));
     *out_l = __popc(__ballot_sync(FULL, ll));
+  }
+}
+
+// ---- TMA bulk copy global -> shared with an mbarrier (cp.async.bulk, SASS UBLKCP) ----
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of dst done
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes) : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+// Wait for phase `parity` of the barrier; bounded so a broken stream traps instead of hanging.
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  for (uint32_t spin = 0;; ++spin) {
+    asm volatile(
+        "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    if (done) return;
+    if (spin > (1u << 28)) __trap();
   }
 }
 
@@ -144,7 +170,10 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   uint32_t* s_diag = s_h128 + 1024;                     // 8 words
   uint32_t* s_priv = s_diag + 8;                        // [warps or 1][pw] counters
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
-  uint2* s_vdesc = reinterpret_cast<uint2*>(s_priv + n_regions * p.pw);  // [warps][128]
+  const uint32_t ob = ((uint32_t)(s_priv + n_regions * p.pw - sm) + 31u) & ~31u;  // 128 B align
+  uint4* s_vbuf = reinterpret_cast<uint4*>(sm + ob);                  // [warps][32 rows][8 x 16 B]
+  uint2* s_vdesc = reinterpret_cast<uint2*>(sm + ob + kWarpsPerCta * 1024);  // [warps][128]
+  uint64_t* s_bar = reinterpret_cast<uint64_t*>(sm + ob + kWarpsPerCta * (1024 + 256));  // [warps]
 
   const uint32_t tid = threadIdx.x;
   for (uint32_t i = tid; i < cap; i += blockDim.x) {
@@ -154,12 +183,17 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
   }
   for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
   for (uint32_t i = tid; i < 2048 + 8 + n_regions * p.pw; i += blockDim.x) s_h32[i] = 0;
+  if (tid < kWarpsPerCta) mbar_init(s_bar + tid, 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
 
   const uint32_t lane = tid & 31u, wib = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   uint32_t* wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
   uint2* vdesc = s_vdesc + wib * 128;
+  uint4* vbuf = s_vbuf + wib * 256;
+  uint64_t* vbar = s_bar + wib;
+  uint32_t vphase = 0;
   const uint32_t PB = 4 * p.nb, PV = 4 * p.nb + 4 * p.nm;
   const uint64_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta;
@@ -230,6 +264,10 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       const bool live = known && act != 0;
       c_inv += known && act == 0;
       const uint32_t G = act & m2;  // guard-true (or taken) active lanes
+      // value rows of this batch are contiguous: start the first bulk copy now, so it lands while
+      // the other handlers work on the batch
+      const uint32_t* vsrc = p.val + 32ull * (vrow_b - p.vrow_base);
+      if ((H & SASSI_H_VALUE) && vtot && lane == 0) bulk_load(vbuf, vsrc, 128u * min(vtot, 32u), vbar);
 
       // ---- Case study I: branch divergence (Fig.4) ----
       if (H & SASSI_H_BRANCH) {
@@ -264,22 +302,23 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       }
       // ---- Case study II: memory address divergence (Fig.6), one warp per address row ----
       if (H & SASSI_H_MEMDIV) {
-        uint32_t selm = __ballot_sync(FULL, live && (info & I_MEMDIV) && G != 0);
+        const bool selm_l = live && (info & I_MEMDIV) && G != 0;
+        uint32_t selm = __ballot_sync(FULL, selm_l);
         const uint64_t* abase = p.addr + 32ull * (arow_b - p.arow_base) + lane;
         const uint32_t arel = __popc(ma & lt);
+        uint32_t my_s = 0, my_l = 0;  // results of this lane's own record
         while (selm) {
           uint64_t a[4];
-          uint32_t g[4], mi[4];
+          uint32_t g[4], jj[4];
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             g[k] = 0;
             if (selm) {
               const int j = __ffs(selm) - 1;
               selm &= selm - 1;
-              const uint32_t r = __shfl_sync(FULL, arel, j);
+              jj[k] = j;
               g[k] = __shfl_sync(FULL, G, j);
-              mi[k] = __shfl_sync(FULL, cidx & 0xFFFFu, j);
-              a[k] = ld_nc_u64(abase + 32 * r);
+              a[k] = ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j));
             }
           }
 #pragma unroll
@@ -287,76 +326,72 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
             if (g[k]) {
               uint32_t s, L;
               memdiv_row(a[k], g[k], lane, &s, &L);
-              const uint32_t n = __popc(g[k]);
-              if (lane < 2)
-                atomicAdd(lane == 0 ? s_h32 + 32 * (n - 1) + (s - 1) : s_h128 + 32 * (n - 1) + (L - 1), 1u);
-              uint32_t* q = wpriv + PB + 4 * mi[k];
-              if (p.priv) {
-                if (lane == 0) {
-                  uint4 c = *reinterpret_cast<uint4*>(q);
-                  c.x += 1;
-                  c.y += n;
-                  c.z += s;
-                  c.w += L;
-                  *reinterpret_cast<uint4*>(q) = c;
-                }
-              } else if (lane >= 2 && lane < 6) {
-                atomicAdd(q + (lane - 2), lane == 2 ? 1u : (lane == 3 ? n : (lane == 4 ? s : L)));
+              if (lane == jj[k]) {
+                my_s = s;
+                my_l = L;
               }
             }
           }
         }
+        // one vectorised update for the batch: each record's lane adds its own results
+        const uint32_t n = __popc(G);
+        if (selm_l) {
+          atomicAdd(s_h32 + 32 * (n - 1) + (my_s - 1), 1u);
+          atomicAdd(s_h128 + 32 * (n - 1) + (my_l - 1), 1u);
+        }
+        add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv, p.priv,
+                      lane);
       }
-      // ---- Case study III: value profiling (Fig.9), 4 value rows per 128-bit warp load ----
+      // ---- Case study III: value profiling (Fig.9): row-per-lane fold of TMA-staged rows ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
         add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
                       p.priv, lane);
         const uint32_t vd0 = info >> I_VD0_SHIFT;
-        for (uint32_t d = 0; d < nd; ++d) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
+#pragma unroll
+        for (uint32_t d = 0; d < 4; ++d)
+          if (d < nd) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
         __syncwarp();
-        // quad q = rows 4q..4q+3 of this batch; lane holds row 4q + lane/8, columns 4*(lane%8)..+3
-        const uint4* vq = reinterpret_cast<const uint4*>(p.val + 32ull * (vrow_b - p.vrow_base)) + lane;
-        const uint32_t nq = (vtot + 3) >> 2;
-        const uint32_t sh = (lane & 7u) * 4;
-        for (uint32_t q0 = 0; q0 < nq; q0 += 4) {
-          uint4 x[4];
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const uint32_t rr = 4 * (q0 + k) + (lane >> 3);
-            x[k] = rr < vtot ? ld_nc_v4(vq + 32 * (q0 + k)) : make_uint4(0, 0, 0, 0);
+        for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
+          const uint32_t nr = min(vtot - s0, 32u);
+          if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
+            __syncwarp();
+            if (lane == 0) bulk_load(vbuf, vsrc + 32ull * s0, 128u * nr, vbar);
           }
+          mbar_wait(vbar, vphase);
+          vphase ^= 1u;
+          const uint2 ds = lane < nr ? vdesc[s0 + lane] : make_uint2(0u, 0u);
+          const uint32_t V = ds.x;
+          // lane folds row s0+lane: 8 chunks of 4 values, chunk order rotated by lane so the 8 lanes
+          // of each shared-memory phase hit 8 different bank groups
+          const uint4* row = vbuf + 8 * lane;
+          uint32_t va = FULL, vo = 0;
+          if (__all_sync(FULL, V == FULL || V == 0)) {
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            if (q0 + k < nq) {
-              const uint32_t rr = 4 * (q0 + k) + (lane >> 3);
-              const uint2 ds = rr < vtot ? vdesc[rr] : make_uint2(0u, 0u);
-              const uint32_t vb = (ds.x >> sh) & 0xFu;
-              uint32_t va, vo;
-              if (__all_sync(FULL, vb == 0xFu || ds.x == 0)) {
-                va = x[k].x & x[k].y & x[k].z & x[k].w;
-                vo = x[k].x | x[k].y | x[k].z | x[k].w;
-              } else {
-                const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
-                const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - (vb >> 3);
-                va = (x[k].x | ~m0) & (x[k].y | ~m1) & (x[k].z | ~m2_) & (x[k].w | ~m3);
-                vo = (x[k].x & m0) | (x[k].y & m1) | (x[k].z & m2_) | (x[k].w & m3);
-              }
-              va &= __shfl_xor_sync(FULL, va, 1);
-              vo |= __shfl_xor_sync(FULL, vo, 1);
-              va &= __shfl_xor_sync(FULL, va, 2);
-              vo |= __shfl_xor_sync(FULL, vo, 2);
-              va &= __shfl_xor_sync(FULL, va, 4);
-              vo |= __shfl_xor_sync(FULL, vo, 4);
-              if ((lane & 7u) == 0 && ds.x != 0) {
-                uint4* st = s_vstate + ds.y;
-                const uint4 c = *st;
-                const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
-                if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
-                if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
-                if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
-              }
+            for (uint32_t k = 0; k < 8; ++k) {
+              const uint4 x = row[(k + lane) & 7u];
+              va &= x.x & x.y & x.z & x.w;
+              vo |= x.x | x.y | x.z | x.w;
             }
+          } else {
+#pragma unroll
+            for (uint32_t k = 0; k < 8; ++k) {
+              const uint32_t c = (k + lane) & 7u;
+              const uint4 x = row[c];
+              const uint32_t vb = V >> (4 * c);
+              const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
+              const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - ((vb >> 3) & 1u);
+              va &= (x.x | ~m0) & (x.y | ~m1) & (x.z | ~m2_) & (x.w | ~m3);
+              vo |= (x.x & m0) | (x.y & m1) | (x.z & m2_) | (x.w & m3);
+            }
+          }
+          if (V != 0) {
+            uint4* st = s_vstate + ds.y;
+            const uint4 c = *st;
+            const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
+            if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
+            if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
+            if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
           }
         }
         __syncwarp();
@@ -476,8 +511,9 @@ KernelFn select_kernel(uint32_t mask) {
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   size_t words = (3ull * c->cap + 3) & ~3ull;
   words += 4ull * c->nvd + 2048 + 8 + (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
-  words = (words + 1) & ~1ull;  // 8-byte align the descriptor area
-  *bytes = 4 * words + sizeof(uint2) * 128 * kWarpsPerCta;
+  words = (words + 31) & ~31ull;                       // 128 B-aligned value-row buffers
+  words += kWarpsPerCta * (1024 + 256 + 2);            // rows (4 KB) + descriptors + mbarrier
+  *bytes = 4 * words;
   return 0;
 }
 
