@@ -15,7 +15,7 @@ constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr uint32_t EMPTY_KEY = 0xFFFFFFFFu;
 constexpr int kConsumeThreads = 256;          // 8 warps per CTA
 constexpr int kWarpsPerCta = kConsumeThreads / 32;
-constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 30;  // keeps every smem u32 partial < 2^32
+constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 29;  // 32-bit record / row indices in a launch
 
 // Packed per-site info word in the hash (bit layout). The companion cidx word holds the
 // site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).
@@ -42,14 +42,14 @@ struct Offsets {
 
 // Kernel parameter block of the fused consume kernel.
 struct ConsumeParams {
-  const uint4* hdr;                 // [n] headers (16 B each)
+  const uint4* hdr;                 // [n] headers (16 B each), this launch's first record first
   const uint64_t* addr;             // addr rows; row r at addr + 32 * (r - arow_base)
   const uint32_t* val;              // val rows;  row r at val + 32 * (r - vrow_base)
   const ulonglong2* cb;             // chunk index for the records of this launch
-  uint64_t n;                       // records in this launch (hdr[0] starts a chunk)
+  uint32_t n;                       // records in this launch (hdr[0] starts a chunk)
   uint64_t arow_base, vrow_base;    // row index of addr[0] / val[0]
   uint64_t arow_end, vrow_end;      // one past the last valid row index (bounds check)
-  const uint32_t* hash;             // [3][cap]: keys, info, cidx
+  const uint4* hash;                // [cap] {key, info, cidx, 0}
   uint32_t cap;                     // power of two
   uint32_t nb, nm, nv, nvd;         // branch sites, memdiv sites, value sites, value (site,dst)s
   uint32_t pw;                      // private counter words per warp (16 B multiple)
@@ -75,7 +75,7 @@ struct sassi_ctx {
   uint64_t checksum = 0;
   // device state
   uint64_t* d_table = nullptr;
-  uint32_t* d_hash = nullptr;       // [3][cap]
+  uint4* d_hash = nullptr;          // [cap] {key, info, cidx, 0}
   uint32_t cap = 0;
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v

@@ -155,54 +155,51 @@ __device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, 
   }
 }
 
+// Shared-memory layout (u32 words). Fixed-size regions first so their offsets are constants.
+constexpr uint32_t kSmH32 = 0;                                      // [32][32] u32
+constexpr uint32_t kSmH128 = 1024;                                  // [32][32] u32
+constexpr uint32_t kSmDiag = 2048;                                  // 8 u32
+constexpr uint32_t kSmBar = 2056;                                   // [warps] u64 mbarriers
+constexpr uint32_t kSmVbuf = 2080;                                  // [warps][32 rows][32 u32]
+constexpr uint32_t kVbufWords = 1024;                               // 4 KB per warp
+constexpr uint32_t kSmVdesc = kSmVbuf + kWarpsPerCta * kVbufWords;  // [warps][128] uint2
+constexpr uint32_t kSmVar = kSmVdesc + kWarpsPerCta * 256;          // hash, vstate, counters
+static_assert(kSmVbuf % 32 == 0 && kSmVar % 4 == 0, "alignment");
+
 template <uint32_t H>
-__global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeParams p) {
-  extern __shared__ __align__(16) uint32_t sm[];
+__global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const ConsumeParams p) {
+  extern __shared__ __align__(128) uint32_t sm[];
   const uint32_t cap = p.cap;
-  uint32_t* s_keys = sm;
-  uint32_t* s_info = sm + cap;
-  uint32_t* s_cidx = sm + 2 * cap;
-  uint32_t o = (3 * cap + 3) & ~3u;
-  uint4* s_vstate = reinterpret_cast<uint4*>(sm + o);  // [nvd]: ones, zeros, isScalar, -
-  o += 4 * p.nvd;
-  uint32_t* s_h32 = sm + o;                             // [32][32]
-  uint32_t* s_h128 = s_h32 + 1024;                      // [32][32]
-  uint32_t* s_diag = s_h128 + 1024;                     // 8 words
-  uint32_t* s_priv = s_diag + 8;                        // [warps or 1][pw] counters
+  uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
+  uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
+  uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + p.nvd); // [warps or 1][pw] counters
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
-  const uint32_t ob = ((uint32_t)(s_priv + n_regions * p.pw - sm) + 31u) & ~31u;  // 128 B align
-  uint4* s_vbuf = reinterpret_cast<uint4*>(sm + ob);                  // [warps][32 rows][8 x 16 B]
-  uint2* s_vdesc = reinterpret_cast<uint2*>(sm + ob + kWarpsPerCta * 1024);  // [warps][128]
-  uint64_t* s_bar = reinterpret_cast<uint64_t*>(sm + ob + kWarpsPerCta * (1024 + 256));  // [warps]
 
   const uint32_t tid = threadIdx.x;
-  for (uint32_t i = tid; i < cap; i += blockDim.x) {
-    s_keys[i] = p.hash[i];
-    s_info[i] = p.hash[cap + i];
-    s_cidx[i] = p.hash[2 * cap + i];
-  }
+  for (uint32_t i = tid; i < cap; i += blockDim.x) s_hash[i] = p.hash[i];
   for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
-  for (uint32_t i = tid; i < 2048 + 8 + n_regions * p.pw; i += blockDim.x) s_h32[i] = 0;
-  if (tid < kWarpsPerCta) mbar_init(s_bar + tid, 1);
+  for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
+  for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;
+  if (tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
 
   const uint32_t lane = tid & 31u, wib = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
-  uint32_t* wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
-  uint2* vdesc = s_vdesc + wib * 128;
-  uint4* vbuf = s_vbuf + wib * 256;
-  uint64_t* vbar = s_bar + wib;
+  uint32_t* const wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
+  uint2* const vdesc = reinterpret_cast<uint2*>(sm + kSmVdesc) + wib * 128;
+  uint4* const vbuf = reinterpret_cast<uint4*>(sm + kSmVbuf + wib * kVbufWords);
+  uint64_t* const vbar = reinterpret_cast<uint64_t*>(sm + kSmBar) + wib;
   uint32_t vphase = 0;
   const uint32_t PB = 4 * p.nb, PV = 4 * p.nb + 4 * p.nm;
-  const uint64_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
-  const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta;
+  const uint32_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
+  const uint32_t nw = gridDim.x * kWarpsPerCta;
   uint32_t c_rec = 0, c_inv = 0, c_unk = 0, c_bad = 0;
   uint32_t acc = 0, acc_w = FULL;  // per-thread-count accumulator of trace warp acc_w, lane = lane
   uint32_t err = 0;
   unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
 
-  for (uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
+  for (uint32_t u = blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
     const ulonglong2 cb0 = p.cb[u];
     const ulonglong2 cb1 = p.cb[u + 1];
     if (!(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end && cb0.y >= p.vrow_base &&
@@ -210,42 +207,38 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       err |= 8u;  // chunk index outside the row buffers
       continue;
     }
-    uint64_t arow = cb0.x, vrow = cb0.y;
-    const uint64_t rec0 = u * SASSI_CHUNK;
-    const uint64_t left = p.n - rec0;
-    const uint32_t nbat = left >= SASSI_CHUNK ? SASSI_CHUNK / 32 : (uint32_t)((left + 31) / 32);
-    uint4 hnext = (rec0 + lane < p.n) ? ld_nc_v4(p.hdr + rec0 + lane) : make_uint4(EMPTY_KEY, 0, 0, 0);
+    // rows are addressed relative to this chunk: 32-bit offsets from here on
+    const uint64_t* const achunk = p.addr + ((cb0.x - p.arow_base) << 5);
+    const uint32_t* const vchunk = p.val + ((cb0.y - p.vrow_base) << 5);
+    const uint32_t aend = (uint32_t)(cb1.x - cb0.x), vend = (uint32_t)(cb1.y - cb0.y);
+    uint32_t arow = 0, vrow = 0;
+    const uint4* const hchunk = p.hdr + u * SASSI_CHUNK;
+    const uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
+    const uint32_t nbat = (nrec + 31) >> 5;
+    uint4 hnext = lane < nrec ? ld_nc_v4(hchunk + lane) : make_uint4(EMPTY_KEY, 0, 0, 0);
     uint32_t b = 0;
     for (; b < nbat; ++b) {
-      const uint64_t i = rec0 + 32 * b + lane;
-      const bool valid = i < p.n;
+      const uint32_t ib = 32 * b + lane;
+      const bool valid = ib < nrec;
       const uint4 h = hnext;
-      if (b + 1 < nbat) {
-        const uint64_t i2 = i + 32;
-        hnext = i2 < p.n ? ld_nc_v4(p.hdr + i2) : make_uint4(EMPTY_KEY, 0, 0, 0);
-      }
-      // ---- find(pc): open-addressed, linear probing (Fig.4 l.23, L239) ----
-      uint32_t info = 0, cidx = 0;
-      bool known = false;
+      if (b + 1 < nbat) hnext = ib + 32 < nrec ? ld_nc_v4(hchunk + ib + 32) : make_uint4(EMPTY_KEY, 0, 0, 0);
+      // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239) ----
+      uint4 e = make_uint4(EMPTY_KEY, 0u, 0u, 0u);
       if (valid) {
         uint32_t slot = fmix32(h.x) & (cap - 1);
         for (;;) {
-          const uint32_t k = s_keys[slot];
-          if (k == h.x) {
-            known = true;
-            info = s_info[slot];
-            cidx = s_cidx[slot];
-            break;
-          }
-          if (k == EMPTY_KEY) break;
+          e = s_hash[slot];
+          if (e.x == h.x || e.x == EMPTY_KEY) break;
           slot = (slot + 1) & (cap - 1);
         }
       }
+      const bool known = valid && e.x == h.x && h.x != EMPTY_KEY;  // 0xFFFFFFFF is never registered
+      const uint32_t info = known ? e.y : 0u, cidx = e.z;
       c_rec += valid;
       c_unk += valid && !known;
       // ---- row indices of this batch (rows follow their records) ----
-      const uint32_t ma = __ballot_sync(FULL, known && (info & I_ADDR_ROW));
-      const uint32_t nd = known ? (info >> I_NDST_SHIFT) & 7u : 0u;
+      const uint32_t ma = __ballot_sync(FULL, info & I_ADDR_ROW);
+      const uint32_t nd = (info >> I_NDST_SHIFT) & 7u;
       uint32_t vpre = 0, vtot = 0;
 #pragma unroll
       for (int k = 0; k < 3; ++k) {
@@ -253,20 +246,20 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
         vpre += __popc(mk & lt) << k;
         vtot += __popc(mk) << k;
       }
-      const uint64_t arow_b = arow, vrow_b = vrow;
+      const uint32_t arow_b = arow, vrow_b = vrow;
       arow += __popc(ma);
       vrow += vtot;
-      if (arow > cb1.x || vrow > cb1.y) {
+      if (arow > aend || vrow > vend) {
         err |= 4u;  // rows of this batch run past the chunk's rows: stream inconsistent
         break;
       }
-      const uint32_t act = h.z, m2 = h.w;
+      const uint32_t act = h.z;
       const bool live = known && act != 0;
       c_inv += known && act == 0;
-      const uint32_t G = act & m2;  // guard-true (or taken) active lanes
+      const uint32_t G = act & h.w;  // guard-true (or taken) active lanes
       // value rows of this batch are contiguous: start the first bulk copy now, so it lands while
       // the other handlers work on the batch
-      const uint32_t* vsrc = p.val + 32ull * (vrow_b - p.vrow_base);
+      const uint32_t* const vsrc = vchunk + 32 * vrow_b;
       if ((H & SASSI_H_VALUE) && vtot && lane == 0) bulk_load(vbuf, vsrc, 128u * min(vtot, 32u), vbar);
 
       // ---- Case study I: branch divergence (Fig.4) ----
@@ -304,105 +297,110 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       if (H & SASSI_H_MEMDIV) {
         const bool selm_l = live && (info & I_MEMDIV) && G != 0;
         uint32_t selm = __ballot_sync(FULL, selm_l);
-        const uint64_t* abase = p.addr + 32ull * (arow_b - p.arow_base) + lane;
-        const uint32_t arel = __popc(ma & lt);
-        uint32_t my_s = 0, my_l = 0;  // results of this lane's own record
-        while (selm) {
-          uint64_t a[4];
-          uint32_t g[4], jj[4];
+        if (selm) {
+          const uint64_t* const abase = achunk + 32 * arow_b + lane;
+          const uint32_t arel = __popc(ma & lt);
+          uint32_t my_s = 0, my_l = 0;  // results of this lane's own record
+          do {
+            uint64_t a[4];
+            uint32_t g[4], jj[4];
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            g[k] = 0;
-            if (selm) {
-              const int j = __ffs(selm) - 1;
-              selm &= selm - 1;
-              jj[k] = j;
-              g[k] = __shfl_sync(FULL, G, j);
-              a[k] = ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j));
-            }
-          }
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            if (g[k]) {
-              uint32_t s, L;
-              memdiv_row(a[k], g[k], lane, &s, &L);
-              if (lane == jj[k]) {
-                my_s = s;
-                my_l = L;
+            for (int k = 0; k < 4; ++k) {
+              g[k] = 0;
+              if (selm) {
+                const int j = __ffs(selm) - 1;
+                selm &= selm - 1;
+                jj[k] = j;
+                g[k] = __shfl_sync(FULL, G, j);
+                a[k] = ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j));
               }
             }
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              if (g[k]) {
+                uint32_t s, L;
+                memdiv_row(a[k], g[k], lane, &s, &L);
+                if (lane == jj[k]) {
+                  my_s = s;
+                  my_l = L;
+                }
+              }
+            }
+          } while (selm);
+          // one vectorised update for the batch: each record's lane adds its own results
+          const uint32_t n = __popc(G);
+          if (selm_l) {
+            atomicAdd(sm + kSmH32 + 32 * (n - 1) + (my_s - 1), 1u);
+            atomicAdd(sm + kSmH128 + 32 * (n - 1) + (my_l - 1), 1u);
           }
+          add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv,
+                        p.priv, lane);
         }
-        // one vectorised update for the batch: each record's lane adds its own results
-        const uint32_t n = __popc(G);
-        if (selm_l) {
-          atomicAdd(s_h32 + 32 * (n - 1) + (my_s - 1), 1u);
-          atomicAdd(s_h128 + 32 * (n - 1) + (my_l - 1), 1u);
-        }
-        add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv, p.priv,
-                      lane);
       }
       // ---- Case study III: value profiling (Fig.9): row-per-lane fold of TMA-staged rows ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
         add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
                       p.priv, lane);
-        const uint32_t vd0 = info >> I_VD0_SHIFT;
+        if (vtot) {
+          const uint32_t vd0 = info >> I_VD0_SHIFT;
 #pragma unroll
-        for (uint32_t d = 0; d < 4; ++d)
-          if (d < nd) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
-        __syncwarp();
-        for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
-          const uint32_t nr = min(vtot - s0, 32u);
-          if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
-            __syncwarp();
-            if (lane == 0) bulk_load(vbuf, vsrc + 32ull * s0, 128u * nr, vbar);
-          }
-          mbar_wait(vbar, vphase);
-          vphase ^= 1u;
-          const uint2 ds = lane < nr ? vdesc[s0 + lane] : make_uint2(0u, 0u);
-          const uint32_t V = ds.x;
-          // lane folds row s0+lane: 8 chunks of 4 values, chunk order rotated by lane so the 8 lanes
-          // of each shared-memory phase hit 8 different bank groups
-          const uint4* row = vbuf + 8 * lane;
-          uint32_t va = FULL, vo = 0;
-          if (__all_sync(FULL, V == FULL || V == 0)) {
-#pragma unroll
-            for (uint32_t k = 0; k < 8; ++k) {
-              const uint4 x = row[(k + lane) & 7u];
-              va &= x.x & x.y & x.z & x.w;
-              vo |= x.x | x.y | x.z | x.w;
+          for (uint32_t d = 0; d < 4; ++d)
+            if (d < nd) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
+          __syncwarp();
+          for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
+            const uint32_t nr = min(vtot - s0, 32u);
+            if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
+              __syncwarp();
+              if (lane == 0) bulk_load(vbuf, vsrc + 32 * s0, 128u * nr, vbar);
             }
-          } else {
+            mbar_wait(vbar, vphase);
+            vphase ^= 1u;
+            const uint2 ds = lane < nr ? vdesc[s0 + lane] : make_uint2(0u, 0u);
+            const uint32_t V = ds.x;
+            // lane folds row s0+lane: 8 chunks of 4 values, chunk order rotated by lane so the 8
+            // lanes of each shared-memory phase hit 8 different bank groups
+            const uint4* row = vbuf + 8 * lane;
+            uint32_t va = FULL, vo = 0;
+            if (__all_sync(FULL, V == FULL || V == 0)) {
 #pragma unroll
-            for (uint32_t k = 0; k < 8; ++k) {
-              const uint32_t c = (k + lane) & 7u;
-              const uint4 x = row[c];
-              const uint32_t vb = V >> (4 * c);
-              const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
-              const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - ((vb >> 3) & 1u);
-              va &= (x.x | ~m0) & (x.y | ~m1) & (x.z | ~m2_) & (x.w | ~m3);
-              vo |= (x.x & m0) | (x.y & m1) | (x.z & m2_) | (x.w & m3);
+              for (uint32_t k = 0; k < 8; ++k) {
+                const uint4 x = row[(k + lane) & 7u];
+                va &= x.x & x.y & x.z & x.w;
+                vo |= x.x | x.y | x.z | x.w;
+              }
+            } else {
+#pragma unroll
+              for (uint32_t k = 0; k < 8; ++k) {
+                const uint32_t c = (k + lane) & 7u;
+                const uint4 x = row[c];
+                const uint32_t vb = V >> (4 * c);
+                const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
+                const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - ((vb >> 3) & 1u);
+                va &= (x.x | ~m0) & (x.y | ~m1) & (x.z | ~m2_) & (x.w | ~m3);
+                vo |= (x.x & m0) | (x.y & m1) | (x.z & m2_) | (x.w & m3);
+              }
+            }
+            if (V != 0) {
+              uint4* st = s_vstate + ds.y;
+              const uint4 c = *st;
+              const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
+              if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
+              if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
+              if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
             }
           }
-          if (V != 0) {
-            uint4* st = s_vstate + ds.y;
-            const uint4 c = *st;
-            const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
-            if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
-            if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
-            if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
-          }
+          __syncwarp();
         }
-        __syncwarp();
       }
     }
-    if (b == nbat && lane == 0 && (arow != cb1.x || vrow != cb1.y)) err |= 4u;  // index disagrees
+    if (b == nbat && lane == 0 && (arow != aend || vrow != vend)) err |= 4u;  // index disagrees
   }
   if (H & SASSI_H_INSTCOUNT) {
     if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
   }
   // ---- diagnostics: warp-reduce, one smem atomic per warp ----
+  uint32_t* const s_diag = sm + kSmDiag;
   c_rec = __reduce_add_sync(FULL, c_rec);
   c_inv = __reduce_add_sync(FULL, c_inv);
   c_unk = __reduce_add_sync(FULL, c_unk);
@@ -453,7 +451,7 @@ __global__ void __launch_bounds__(kConsumeThreads) consume_kernel(const ConsumeP
       atomicAdd(g + 3, (unsigned long long)t.w);
     }
     for (uint32_t c = tid; c < 2048; c += blockDim.x) {
-      const uint32_t v = s_h32[c];
+      const uint32_t v = sm[kSmH32 + c];
       if (v) atomicAdd(table + (c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024)), (unsigned long long)v);
     }
   }
@@ -509,10 +507,7 @@ KernelFn select_kernel(uint32_t mask) {
 }  // namespace
 
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
-  size_t words = (3ull * c->cap + 3) & ~3ull;
-  words += 4ull * c->nvd + 2048 + 8 + (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
-  words = (words + 31) & ~31ull;                       // 128 B-aligned value-row buffers
-  words += kWarpsPerCta * (1024 + 256 + 2);            // rows (4 KB) + descriptors + mbarrier
+  size_t words = kSmVar + 4ull * c->cap + 4ull * c->nvd + (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
   *bytes = 4 * words;
   return 0;
 }
@@ -525,7 +520,7 @@ int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
   SASSI_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kConsumeThreads, c->smem_bytes));
   if (per_sm < 1) return set_error(SASSI_ENOSPC, "consume kernel does not fit on an SM");
   c->ctas_per_sm = per_sm;
-  const uint64_t units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
+  const uint64_t units = ((uint64_t)p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
   uint64_t grid = (uint64_t)c->num_sms * per_sm;
   const uint64_t need = (units + kWarpsPerCta - 1) / kWarpsPerCta;
   if (grid > need) grid = need ? need : 1;

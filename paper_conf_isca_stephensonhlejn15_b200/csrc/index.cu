@@ -8,7 +8,7 @@ namespace {
 
 // one warp per chunk: per-chunk addr-row and val-row counts
 __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restrict__ hdr, uint64_t n,
-                                                           const uint32_t* __restrict__ hash,
+                                                           const uint4* __restrict__ hash,
                                                            uint32_t cap, uint64_t* na, uint64_t* nv) {
   const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
@@ -21,9 +21,10 @@ __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restri
     const uint32_t pc = hdr[i].x;
     uint32_t slot = fmix32(pc) & (cap - 1);
     for (;;) {
-      const uint32_t key = hash[slot];
+      const uint4 e = hash[slot];
+      const uint32_t key = e.x;
       if (key == pc) {
-        const uint32_t inf = hash[cap + slot];
+        const uint32_t inf = e.y;
         a += (inf & I_ADDR_ROW) ? 1u : 0u;
         v += (inf >> I_NDST_SHIFT) & 7u;
         break;

@@ -48,6 +48,17 @@ def test_random_traces(seed, n):
     assert diff_tables(t, o, len(s), W) is None
 
 
+def test_reserved_pc_record_is_unknown():
+    """A record whose pc is the reserved empty-slot key 0xFFFFFFFF is an unregistered pc."""
+    s, W, hdr, addr, val = random_trace(31337, n=700)
+    hdr = hdr.copy()
+    hdr["pc"][::7] = np.where(np.isin(hdr["pc"][::7], s["pc"]), hdr["pc"][::7], 0xFFFFFFFF)
+    o = oracle.run(s, W, oracle.H_ALL, hdr, addr, val)
+    assert int(oracle.sections(o, len(s), W)["diag"][2]) > 0
+    t = gpu_table(s, W, sassi.SASSI_H_ALL, to_device(s, hdr, addr, val))
+    assert diff_tables(t, o, len(s), W) is None
+
+
 def test_empty_stream():
     s = T0.sites()
     hdr, addr, val = T0.records()
