@@ -162,12 +162,11 @@ constexpr uint32_t kSmDiag = 2048;                                  // 8 u32
 constexpr uint32_t kSmBar = 2056;                                   // [warps] u64 mbarriers
 constexpr uint32_t kSmVbuf = 2080;                                  // [warps][32 rows][32 u32]
 constexpr uint32_t kVbufWords = 1024;                               // 4 KB per warp
-constexpr uint32_t kSmVdesc = kSmVbuf + kWarpsPerCta * kVbufWords;  // [warps][128] uint2
-constexpr uint32_t kSmVar = kSmVdesc + kWarpsPerCta * 256;          // hash, vstate, counters
+constexpr uint32_t kSmVar = kSmVbuf + kWarpsPerCta * kVbufWords;    // hash, vstate, counters
 static_assert(kSmVbuf % 32 == 0 && kSmVar % 4 == 0, "alignment");
 
 template <uint32_t H>
-__global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const ConsumeParams p) {
+__global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
   const uint32_t cap = p.cap;
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
@@ -187,7 +186,6 @@ __global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const Consu
   const uint32_t lane = tid & 31u, wib = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   uint32_t* const wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
-  uint2* const vdesc = reinterpret_cast<uint2*>(sm + kSmVdesc) + wib * 128;
   uint4* const vbuf = reinterpret_cast<uint4*>(sm + kSmVbuf + wib * kVbufWords);
   uint64_t* const vbar = reinterpret_cast<uint64_t*>(sm + kSmBar) + wib;
   uint32_t vphase = 0;
@@ -343,11 +341,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const Consu
         add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
                       p.priv, lane);
         if (vtot) {
-          const uint32_t vd0 = info >> I_VD0_SHIFT;
-#pragma unroll
-          for (uint32_t d = 0; d < 4; ++d)
-            if (d < nd) vdesc[vpre + d] = make_uint2(selv ? G : 0u, vd0 + d);
-          __syncwarp();
+          const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
+          const uint32_t vslot = info >> I_VD0_SHIFT;         // its first value-state slot
           for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
             const uint32_t nr = min(vtot - s0, 32u);
             if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
@@ -356,8 +351,16 @@ __global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const Consu
             }
             mbar_wait(vbar, vphase);
             vphase ^= 1u;
-            const uint2 ds = lane < nr ? vdesc[s0 + lane] : make_uint2(0u, 0u);
-            const uint32_t V = ds.x;
+            // owner of row r = s0 + lane: the largest lane j with vpre_j <= r (always one with a
+            // value row, since a lane without rows shares vpre with its successor)
+            const uint32_t r = s0 + lane;
+            uint32_t j = 0;
+#pragma unroll
+            for (uint32_t step = 16; step; step >>= 1)
+              if (__shfl_sync(FULL, vpre, j + step) <= r) j += step;
+            const uint32_t Vj = __shfl_sync(FULL, vsel, j);
+            const uint32_t slot = __shfl_sync(FULL, vslot, j) + (r - __shfl_sync(FULL, vpre, j));
+            const uint32_t V = lane < nr ? Vj : 0u;
             // lane folds row s0+lane: 8 chunks of 4 values, chunk order rotated by lane so the 8
             // lanes of each shared-memory phase hit 8 different bank groups
             const uint4* row = vbuf + 8 * lane;
@@ -382,7 +385,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 3) consume_kernel(const Consu
               }
             }
             if (V != 0) {
-              uint4* st = s_vstate + ds.y;
+              uint4* st = s_vstate + slot;
               const uint4 c = *st;
               const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
               if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
