@@ -50,10 +50,28 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
   return x;
 }
 
+// Bitonic sort of one key per lane across the warp (ascending in lane order).
+template <typename T>
+__device__ __forceinline__ T warp_sort(T v, uint32_t lane) {
+#pragma unroll
+  for (uint32_t k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+    for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+      const T o = __shfl_xor_sync(FULL, v, j);
+      const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0);
+      v = keep_min ? (o < v ? o : v) : (o > v ? o : v);
+    }
+  }
+  return v;
+}
+
 // Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
-// over the lanes of G. Fast path when every sector lies within [-32, 31] of the first G lane's (same
-// high word): a 64-bit window bitmap OR-reduced across the warp (REDUX). Otherwise MATCH.ANY groups
-// equal keys and the group leaders are counted.
+// over the lanes of G (the count of Fig.6's leader-election loop, l.16-26).
+//  - window path: every sector within [-32, 31] of the first G lane's (same high word): a 64-bit
+//    window bitmap OR-reduced across the warp (REDUX), popcount.
+//  - otherwise: sort the keys across the warp (bitonic, 32-bit when all high words agree) with the
+//    lanes outside G padded to the maximum so they sort last, and count positions < n whose key
+//    differs from the previous one; lines come from the same sorted sectors (>> 2 keeps order).
 __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
                                            uint32_t* out_l) {
   const bool in = (G >> lane) & 1u;
@@ -62,23 +80,30 @@ __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane
   const int leader = __ffs(G) - 1;
   const uint32_t blo = __shfl_sync(FULL, slo, leader), bhi = __shfl_sync(FULL, shi, leader);
   const uint32_t e = slo - blo + 32u;  // window position, valid when < 64 and high words agree
-  if (__all_sync(FULL, !in || (e < 64u && shi == bhi))) {
+  const bool same_hi = !in || shi == bhi;
+  if (__all_sync(FULL, same_hi && (!in || e < 64u))) {
     const uint32_t lo = __reduce_or_sync(FULL, in ? (1u << e) : 0u);          // e >= 32 -> 0
     const uint32_t hi = __reduce_or_sync(FULL, in ? (1u << (e - 32u)) : 0u);  // e < 32 -> 0
     const uint32_t ln = (uint32_t)(((int32_t)(e - 32u) + (int32_t)(blo & 3u)) >> 2) + 8u;  // 0..16
     *out_s = __popc(lo) + __popc(hi);
     *out_l = __popc(__reduce_or_sync(FULL, in ? (1u << ln) : 0u));
-  } else {
-    uint32_t gs = 0, gl = 0;
-    if (in) {
-      gs = __match_any_sync(G, sec);
-      gl = __match_any_sync(G, sec >> 2);
-    }
-    const bool ls = in && (uint32_t)(__ffs(gs) - 1) == lane;
-    const bool ll = in && (uint32_t)(__ffs(gl) - 1) == lane;
-    *out_s = __popc(__ballot_sync(FULL, ls));
-    *out_l = __popc(__ballot_sync(FULL, ll));
+    return;
   }
+  const uint32_t n = __popc(G);
+  bool new_s, new_l;
+  if (__all_sync(FULL, same_hi)) {
+    const uint32_t v = warp_sort<uint32_t>(in ? slo : FULL, lane);
+    const uint32_t pv = __shfl_up_sync(FULL, v, 1);
+    new_s = lane < n && (lane == 0 || v != pv);
+    new_l = lane < n && (lane == 0 || (v >> 2) != (pv >> 2));
+  } else {
+    const uint64_t v = warp_sort<uint64_t>(in ? sec : ~0ull, lane);
+    const uint64_t pv = __shfl_up_sync(FULL, v, 1);
+    new_s = lane < n && (lane == 0 || v != pv);
+    new_l = lane < n && (lane == 0 || (v >> 2) != (pv >> 2));
+  }
+  *out_s = __popc(__ballot_sync(FULL, new_s));
+  *out_l = __popc(__ballot_sync(FULL, new_l));
 }
 
 // ---- TMA bulk copy global -> shared with an mbarrier (cp.async.bulk, SASS UBLKCP) ----
