@@ -246,3 +246,21 @@ def test_consume_host_equals_device():
     ctx.consume_host(hrec)
     assert np.array_equal(ctx.read_tables(), t_dev)
     ctx.close()
+
+
+def test_merge_single_rank_nccl():
+    """sassi_merge through a real 1-rank NCCL communicator: pack -> ncclAllReduce -> unpack must
+    leave the tables unchanged (sums over one rank; masks survive the byte-expansion round trip)."""
+    s, W, hdr, addr, val = random_trace(555, n=6000)
+    d = to_device(s, hdr, addr, val)
+    ctx = sassi.Context(s, W, sassi.SASSI_H_ALL)
+    ctx.consume(d)
+    before = ctx.read_tables()
+    uid = sassi.sassi_nccl_get_unique_id()
+    comm = sassi.sassi_nccl_comm_create(1, 0, uid, torch.cuda.current_device())
+    ctx.merge(comm)
+    after = ctx.read_tables()
+    sassi.sassi_nccl_comm_destroy(comm)
+    ctx.close()
+    assert np.array_equal(after, before)
+    assert np.array_equal(after, oracle.run(s, W, oracle.H_ALL, hdr, addr, val))
