@@ -185,10 +185,11 @@ constexpr uint32_t kSmH32 = 0;                                      // [32][32] 
 constexpr uint32_t kSmH128 = 1024;                                  // [32][32] u32
 constexpr uint32_t kSmDiag = 2048;                                  // 8 u32
 constexpr uint32_t kSmBar = 2056;                                   // [warps] u64 mbarriers
-constexpr uint32_t kSmVbuf = 2080;                                  // [warps][32 rows][32 u32]
+constexpr uint32_t kSmVbuf = (kSmBar + 2 * kWarpsPerCta + 31) & ~31u;  // [warps][32 rows][32 u32]
 constexpr uint32_t kVbufWords = 1024;                               // 4 KB per warp
 constexpr uint32_t kSmVar = kSmVbuf + kWarpsPerCta * kVbufWords;    // hash, vstate, counters
-static_assert(kSmVbuf % 32 == 0 && kSmVar % 4 == 0, "alignment");
+static_assert(kSmVbuf % 32 == 0 && kSmVar % 4 == 0 && kSmVbuf >= kSmBar + 2 * kWarpsPerCta,
+              "shared-memory layout");
 
 template <uint32_t H>
 __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const ConsumeParams p) {
