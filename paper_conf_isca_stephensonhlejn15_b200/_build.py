@@ -44,7 +44,7 @@ def build(force: bool = False, verbose: bool = False) -> dict:
     # product library
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
     deps = srcs + glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h")) + \
-        [os.path.join(INCLUDE, "sassi.h")]
+        glob.glob(os.path.join(INCLUDE, "*.h"))
     tgt = os.path.join(LIB, "libsassi.so")
     if srcs and (force or _stale(tgt, deps)):
         from concurrent.futures import ThreadPoolExecutor

@@ -24,8 +24,10 @@ SASSI_OK, SASSI_EINVAL, SASSI_ECUDA, SASSI_ENCCL = 0, -1, -2, -3
 SASSI_ENOSPC, SASSI_ESTATE, SASSI_EMISMATCH, SASSI_EFORMAT = -4, -5, -6, -7
 SASSI_H_BRANCH, SASSI_H_MEMDIV, SASSI_H_VALUE, SASSI_H_INSTCOUNT, SASSI_H_ALL = 1, 2, 4, 8, 15
 SASSI_CHUNK = 256
+SASSI_IK_VECADD, SASSI_IK_BFS, SASSI_IK_SGEMM, SASSI_IK_STENCIL = 0, 1, 2, 3
+SASSI_IK_NONE, SASSI_IK_TRACE, SASSI_IK_NULL_ABI = 0, 16, 32
 
-# every function declared in include/sassi.h: name -> (restype, argtypes)
+# every function declared in include/*.h: name -> (restype, argtypes)
 _vp, _u32, _u64, _i = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
 
 
@@ -56,6 +58,13 @@ SIGNATURES = {
     "sassi_nccl_comm_create": (_i, [ctypes.POINTER(_vp), _i, _i, _vp, _i]),
     "sassi_nccl_comm_destroy": (_i, [_vp]),
     "sassi_kernel_launches": (_i, [_vp, ctypes.POINTER(_u64)]),
+    "sassi_ik_create": (_i, [ctypes.POINTER(_vp), _i, _u32, _u64, _i]),
+    "sassi_ik_destroy": (None, [_vp]),
+    "sassi_ik_sites": (_i, [_vp, _vp, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32)]),
+    "sassi_ik_run": (_i, [_vp, _u32, _vp, _vp]),
+    "sassi_ik_trace_totals": (_i, [_vp, ctypes.POINTER(_u64), ctypes.POINTER(_u64), ctypes.POINTER(_u64)]),
+    "sassi_ik_trace_copy": (_i, [_vp, _vp, _vp, _vp, _vp]),
+    "sassi_ik_output_checksum": (_i, [_vp, ctypes.POINTER(_u64)]),
     "sassi_strerror": (ctypes.c_char_p, [_i]),
     "sassi_last_error": (ctypes.c_char_p, []),
 }
@@ -264,6 +273,94 @@ class Context:
     def close(self):
         if self.handle:
             sassi_ctx_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ---- instrumented synthetic kernels (include/sassi_ik.h) ---------------------------------------
+def sassi_ik_create(kernel: int, size: int = 0, seed: int = 20150613, device: int = 0) -> int:
+    h = _vp()
+    _check(lib().sassi_ik_create(ctypes.byref(h), kernel, size, seed, device))
+    return h.value
+
+
+def sassi_ik_destroy(ik: int) -> None:
+    lib().sassi_ik_destroy(ik)
+
+
+def sassi_ik_sites(ik: int):
+    n, w = _u32(), _u32()
+    _check(lib().sassi_ik_sites(ik, None, 0, ctypes.byref(n), ctypes.byref(w)))
+    out = np.zeros(n.value, dtype=SITE_DTYPE)
+    _check(lib().sassi_ik_sites(ik, out.ctypes.data, n.value, ctypes.byref(n), ctypes.byref(w)))
+    return out, w.value
+
+
+def sassi_ik_run(ik: int, mode: int, ctx: int | None = None, stream=None) -> None:
+    _check(lib().sassi_ik_run(ik, mode, ctx, _stream(stream)))
+
+
+def sassi_ik_trace_totals(ik: int):
+    a, b, c = _u64(), _u64(), _u64()
+    _check(lib().sassi_ik_trace_totals(ik, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c)))
+    return a.value, b.value, c.value
+
+
+def sassi_ik_trace_copy(ik: int, hdr, addr, val, stream=None) -> None:
+    _check(lib().sassi_ik_trace_copy(ik, _ptr(hdr), _ptr(addr), _ptr(val), _stream(stream)))
+
+
+def sassi_ik_output_checksum(ik: int) -> int:
+    c = _u64()
+    _check(lib().sassi_ik_output_checksum(ik, ctypes.byref(c)))
+    return c.value
+
+
+class InstrumentedKernel:
+    """A synthetic kernel with hand-placed SASSI sites (vecadd / bfs / sgemm / stencil)."""
+
+    NAMES = {"vecadd": SASSI_IK_VECADD, "bfs": SASSI_IK_BFS, "sgemm": SASSI_IK_SGEMM,
+             "stencil": SASSI_IK_STENCIL}
+
+    def __init__(self, kernel, size: int = 0, seed: int = 20150613, device: int = 0):
+        kid = self.NAMES[kernel] if isinstance(kernel, str) else kernel
+        self.handle = sassi_ik_create(kid, size, seed, device)
+        self.device = device
+        self.sites, self.n_warps = sassi_ik_sites(self.handle)
+
+    def context(self, handlers: int = SASSI_H_ALL) -> Context:
+        return Context(self.sites, self.n_warps, handlers, self.device)
+
+    def run(self, mode: int, ctx: Context | None = None, stream=None) -> None:
+        sassi_ik_run(self.handle, mode, ctx.handle if ctx is not None else None, stream)
+
+    def checksum(self) -> int:
+        return sassi_ik_output_checksum(self.handle)
+
+    def trace(self, ctx: Context, stream=None) -> dict:
+        """Run in trace mode; return the warp-major SRF1 stream as device tensors (+ chunk index)."""
+        import torch
+        sassi_ik_run(self.handle, SASSI_IK_TRACE, None, stream)
+        n, na, nv = sassi_ik_trace_totals(self.handle)
+        dev = torch.device("cuda", self.device)
+        hdr = torch.empty((max(n, 1), 4), dtype=torch.int32, device=dev)
+        addr = torch.empty((max(na, 1), 32), dtype=torch.int64, device=dev)
+        val = torch.empty((max(nv, 1), 32), dtype=torch.int32, device=dev)
+        sassi_ik_trace_copy(self.handle, hdr, addr, val, stream)
+        cb = torch.zeros(((n + SASSI_CHUNK - 1) // SASSI_CHUNK + 1, 2), dtype=torch.int64, device=dev)
+        sassi_index_records(ctx.handle, hdr, n, cb, stream)
+        torch.cuda.synchronize(dev)
+        return dict(hdr=hdr[:n], addr=addr[:na], val=val[:nv], chunk_base=cb, n=n, n_addr_rows=na,
+                    n_val_rows=nv, sites=self.sites)
+
+    def close(self):
+        if self.handle:
+            sassi_ik_destroy(self.handle)
             self.handle = None
 
     def __del__(self):
