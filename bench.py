@@ -42,6 +42,7 @@ def parse():
     ap.add_argument("--workload", default="c3", choices=["c2", "c3", "c4"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-slowdown", action="store_true")
     return ap.parse_args()
 
 
@@ -176,10 +177,11 @@ def run_reference(args, rank, world):
 
 
 def cpu_baseline(args, d_rec, mask, P):
-    """The oracle as it stands, single-threaded, on a ~10-30 s bounded sample (rank 0, N=1)."""
+    """The oracle as it stands, single-threaded, timed for ~10 s on a bounded sample (rank 0, N=1):
+    the first 2^23 records of the same stream, copied to the host, folded repeatedly."""
     import oracle
     from paper_conf_isca_stephensonhlejn15_b200 import gen
-    n = 1 << 22
+    n = min(1 << 23, d_rec["n"] // 256 * 256)
     pre_cb = d_rec["chunk_base"][n // 256].cpu().numpy().view(np.uint64)
     pre = dict(d_rec, hdr=d_rec["hdr"][:n], addr=d_rec["addr"][: int(pre_cb[0])],
                val=d_rec["val"][: int(pre_cb[1])], n=n, n_addr_rows=int(pre_cb[0]),
@@ -191,7 +193,7 @@ def cpu_baseline(args, d_rec, mask, P):
         oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"])
         reps += 1
         el = time.perf_counter() - t0
-        if el > 8.0 or reps >= 3:
+        if el > 10.0 or reps >= 30:
             break
     return {"value": reps * n / el, "unit": "records/s", "cores": 1, "kind": "oracle",
             "sample": "first %d records of the %s stream, %d repetition(s), %.1f s" %
@@ -282,6 +284,10 @@ def main():
     if not args.no_cpu_baseline and rank == 0 and world == 1:
         cpu = cpu_baseline(args, rec, mask, P)
 
+    slow = None
+    if not args.no_slowdown and rank == 0:
+        slow = measure_slowdown(dev)
+
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world,
@@ -313,12 +319,52 @@ def main():
             line["e2e"] = e2e
         if cpu:
             line["cpu_baseline"] = cpu
+        if slow:
+            line["instrumented_slowdown"] = slow
         print(json.dumps(line), flush=True)
     if comm is not None:
         sassi.sassi_nccl_comm_destroy(comm)
     ctx.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def measure_slowdown(dev):
+    """Instrumented-kernel slowdown K = t_instrumented / t_uninstrumented (the K column of the
+    paper's Table 3), median of 5 runs each (L679), per handler, for the four synthetic
+    kernels at their timing sizes; `null_abi` is the paper's stubbed-handler control (L687)."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    modes = {"null_abi": sassi.SASSI_IK_NULL_ABI, "branch": 1, "memdiv": 2, "value": 4,
+             "instcount": 8, "all": 15}
+    out = {}
+    stream = torch.cuda.current_stream(dev)
+    for name in ("vecadd", "bfs", "sgemm", "stencil"):
+        ik = sassi.InstrumentedKernel(name, 0, device=dev.index)
+        ctx = ik.context(sassi.SASSI_H_ALL)
+
+        def timed(mode):
+            ts = []
+            for rep in range(6):
+                if mode & 15:
+                    ctx.reset(stream)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                ik.run(mode, ctx if mode & 15 else None, stream)
+                b.record(stream)
+                b.synchronize()
+                if rep:
+                    ts.append(a.elapsed_time(b))
+            return statistics.median(ts)
+
+        base = timed(sassi.SASSI_IK_NONE)
+        r = {"base_ms": base}
+        for k, m in modes.items():
+            r[k] = timed(m) / base
+        out[name] = r
+        ctx.close()
+        ik.close()
+    return out
 
 
 def measure_e2e(rec, P, mask, n_e2e, dev):
