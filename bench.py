@@ -212,7 +212,9 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    launched = "RANK" in os.environ  # under torchrun (any world size)
+    merge_on = world > 1 or os.environ.get("SASSI_BENCH_FORCE_MERGE") == "1"
+    if launched:
         dist.init_process_group("nccl", device_id=dev)
     P, limit, desc = workload_program(args.workload, world)
     mask = gen.PRESETS[args.workload][2]
@@ -222,11 +224,12 @@ def main():
     alg_bytes, n_glob = algorithmic_bytes(rec, mask)
     ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
     comm = None
-    if world > 1:
+    if merge_on:
         uid = torch.zeros(128, dtype=torch.uint8, device=dev)
         if rank == 0:
             uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
-        dist.broadcast(uid, 0)
+        if launched:
+            dist.broadcast(uid, 0)
         comm = sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
     stream = torch.cuda.current_stream(dev)
     sample = bool(mask & 8)
@@ -246,7 +249,7 @@ def main():
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
-    if world > 1:
+    if launched:
         dist.barrier()
     torch.cuda.synchronize()
     launches0 = ctx.kernel_launches()
@@ -259,13 +262,13 @@ def main():
             step(*evs[k])
         t_end.record(stream)
         torch.cuda.synchronize()
-    if world > 1:
+    if launched:
         dist.barrier()
     torch.cuda.synchronize()
     launches = ctx.kernel_launches() - launches0
     ms = t_start.elapsed_time(t_end)
     consume_ms = [a.elapsed_time(b) for a, b in evs]
-    if world > 1:
+    if launched:
         tt = torch.tensor([ms], device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
@@ -302,7 +305,8 @@ def main():
                        "algorithmic_bytes_per_gpu": alg_bytes,
                        "l2": "inputs (%.1f GB) exceed the 126 MB L2; no flush" % (
                            (16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"]) / 1e9),
-                       "parallelism": "dp%d (warp-id shards, NCCL allreduce merge)" % world},
+                       "parallelism": "dp%d (warp-id shards%s)" % (
+                           world, ", NCCL allreduce merge per step" if merge_on else "")},
             "hbm_gbs": world * alg_bytes * args.steps / sec / 1e9,
             "hbm_frac_of_spec_8tbs": alg_bytes * args.steps / sec / 1e9 / SPEC_HBM_GBS,
             "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
@@ -325,7 +329,7 @@ def main():
     if comm is not None:
         sassi.sassi_nccl_comm_destroy(comm)
     ctx.close()
-    if world > 1:
+    if launched:
         dist.destroy_process_group()
 
 
