@@ -224,10 +224,11 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
   unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
 
   for (uint32_t u = blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
-    const ulonglong2 cb0 = p.cb[u];
-    const ulonglong2 cb1 = p.cb[u + 1];
-    if (!(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end && cb0.y >= p.vrow_base &&
-          cb0.y <= cb1.y && cb1.y <= p.vrow_end)) {
+    constexpr bool kUnitRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
+    const ulonglong2 cb0 = kUnitRows ? p.cb[u] : make_ulonglong2(p.arow_base, p.vrow_base);
+    const ulonglong2 cb1 = kUnitRows ? p.cb[u + 1] : cb0;
+    if (kUnitRows && !(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end &&
+                       cb0.y >= p.vrow_base && cb0.y <= cb1.y && cb1.y <= p.vrow_end)) {
       err |= 8u;  // chunk index outside the row buffers
       continue;
     }
@@ -260,22 +261,28 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       const uint32_t info = known ? e.y : 0u, cidx = e.z;
       c_rec += valid;
       c_unk += valid && !known;
-      // ---- row indices of this batch (rows follow their records) ----
-      const uint32_t ma = __ballot_sync(FULL, info & I_ADDR_ROW);
+      // ---- row indices of this batch (rows follow their records); only handlers that read
+      // payload rows need them, header-only handler sets skip the bookkeeping ----
+      constexpr bool kRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
+      const uint32_t ma = kRows ? __ballot_sync(FULL, info & I_ADDR_ROW) : 0u;
       const uint32_t nd = (info >> I_NDST_SHIFT) & 7u;
       uint32_t vpre = 0, vtot = 0;
+      if (kRows) {
 #pragma unroll
-      for (int k = 0; k < 3; ++k) {
-        const uint32_t mk = __ballot_sync(FULL, (nd >> k) & 1u);
-        vpre += __popc(mk & lt) << k;
-        vtot += __popc(mk) << k;
+        for (int k = 0; k < 3; ++k) {
+          const uint32_t mk = __ballot_sync(FULL, (nd >> k) & 1u);
+          vpre += __popc(mk & lt) << k;
+          vtot += __popc(mk) << k;
+        }
       }
       const uint32_t arow_b = arow, vrow_b = vrow;
-      arow += __popc(ma);
-      vrow += vtot;
-      if (arow > aend || vrow > vend) {
-        err |= 4u;  // rows of this batch run past the chunk's rows: stream inconsistent
-        break;
+      if (kRows) {
+        arow += __popc(ma);
+        vrow += vtot;
+        if (arow > aend || vrow > vend) {
+          err |= 4u;  // rows of this batch run past the chunk's rows: stream inconsistent
+          break;
+        }
       }
       const uint32_t act = h.z;
       const bool live = known && act != 0;
@@ -423,7 +430,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
         }
       }
     }
-    if (b == nbat && lane == 0 && (arow != aend || vrow != vend)) err |= 4u;  // index disagrees
+    if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && lane == 0 && (arow != aend || vrow != vend))
+      err |= 4u;  // index disagrees with the rows
   }
   if (H & SASSI_H_INSTCOUNT) {
     if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
