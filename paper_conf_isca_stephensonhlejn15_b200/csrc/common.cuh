@@ -76,6 +76,9 @@ struct sassi_ctx {
   // device state
   uint64_t* d_table = nullptr;
   uint4* d_hash = nullptr;          // [cap] {key, info, cidx, 0}
+  std::vector<uint4> entries;       // per registered site {pc, info, cidx, 0} (host copy)
+  uint32_t cap_base = 0;            // pow2 >= 2 * n_sites
+  uint32_t hash_cap = 0;            // capacity of the table on the device
   uint32_t cap = 0;
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v

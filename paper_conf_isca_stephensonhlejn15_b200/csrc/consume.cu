@@ -180,32 +180,49 @@ __device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, 
   }
 }
 
-// Shared-memory layout (u32 words). Fixed-size regions first so their offsets are constants.
-constexpr uint32_t kSmH32 = 0;                                      // [32][32] u32
-constexpr uint32_t kSmH128 = 1024;                                  // [32][32] u32
-constexpr uint32_t kSmDiag = 2048;                                  // 8 u32
-constexpr uint32_t kSmBar = 2056;                                   // [warps] u64 mbarriers
-constexpr uint32_t kSmVbuf = (kSmBar + 2 * kWarpsPerCta + 31) & ~31u;  // [warps][32 rows][32 u32]
-constexpr uint32_t kVbufWords = 1024;                               // 4 KB per warp
-constexpr uint32_t kSmVar = kSmVbuf + kWarpsPerCta * kVbufWords;    // hash, vstate, counters
-static_assert(kSmVbuf % 32 == 0 && kSmVar % 4 == 0 && kSmVbuf >= kSmBar + 2 * kWarpsPerCta,
-              "shared-memory layout");
+// Shared-memory layout (u32 words) for handler set H: only the regions the attached handlers use,
+// fixed-size regions first so their offsets are compile-time constants.
+constexpr uint32_t kVbufWords = 1024;  // 4 KB of value rows per warp
+template <uint32_t H>
+struct SmLayout {
+  static constexpr bool kMem = (H & SASSI_H_MEMDIV) != 0, kVal = (H & SASSI_H_VALUE) != 0;
+  static constexpr uint32_t kDiag = 0;                                  // 8 u32
+  static constexpr uint32_t kH32 = 8;                                   // [32][32] u32 (memdiv)
+  static constexpr uint32_t kH128 = kH32 + 1024;                        // [32][32] u32 (memdiv)
+  static constexpr uint32_t kBar = kMem ? kH128 + 1024 : 8;             // [warps] u64 (value)
+  static constexpr uint32_t kVbuf = kVal ? ((kBar + 2 * kWarpsPerCta + 31) & ~31u) : kBar;
+  static constexpr uint32_t kVar = kVbuf + (kVal ? kWarpsPerCta * kVbufWords : 0u);  // hash, ...
+  static_assert(kVbuf % 32 == 0 || !kVal, "value buffers must be 128 B aligned");
+  static_assert(kVar % 4 == 0 && kBar % 2 == 0, "alignment");
+};
+// host mirror of SmLayout<H>::kVar
+uint32_t sm_var_words(uint32_t H) {
+  const bool mem = H & SASSI_H_MEMDIV, val = H & SASSI_H_VALUE;
+  const uint32_t bar = mem ? 8 + 2048 : 8;
+  const uint32_t vbuf = val ? ((bar + 2 * kWarpsPerCta + 31) & ~31u) : bar;
+  return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
+}
 
 template <uint32_t H>
 __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
+  using Ly = SmLayout<H>;
+  constexpr uint32_t kSmDiag = Ly::kDiag, kSmH32 = Ly::kH32, kSmH128 = Ly::kH128, kSmBar = Ly::kBar,
+                     kSmVbuf = Ly::kVbuf, kSmVar = Ly::kVar;
   const uint32_t cap = p.cap;
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
   uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
-  uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + p.nvd); // [warps or 1][pw] counters
+  uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + (Ly::kVal ? p.nvd : 0u));  // counters
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
 
   const uint32_t tid = threadIdx.x;
   for (uint32_t i = tid; i < cap; i += blockDim.x) s_hash[i] = p.hash[i];
-  for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
-  for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
-  for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;
-  if (tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
+  if (Ly::kVal)
+    for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
+  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
+    for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
+  for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
+  if (Ly::kVal && tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
 
@@ -240,21 +257,23 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
     const uint4* const hchunk = p.hdr + u * SASSI_CHUNK;
     const uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
     const uint32_t nbat = (nrec + 31) >> 5;
-    uint4 hnext = lane < nrec ? ld_nc_v4(hchunk + lane) : make_uint4(EMPTY_KEY, 0, 0, 0);
+    // header loads are clamped to the chunk's last record (always in bounds) and masked by `valid`
+    const uint32_t ilast = nrec - 1;
+    uint4 hnext = ld_nc_v4(hchunk + min(lane, ilast));
     uint32_t b = 0;
     for (; b < nbat; ++b) {
       const uint32_t ib = 32 * b + lane;
       const bool valid = ib < nrec;
       const uint4 h = hnext;
-      if (b + 1 < nbat) hnext = ib + 32 < nrec ? ld_nc_v4(hchunk + ib + 32) : make_uint4(EMPTY_KEY, 0, 0, 0);
+      if (b + 1 < nbat) hnext = ld_nc_v4(hchunk + min(ib + 32, ilast));
       // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239) ----
       uint4 e = make_uint4(EMPTY_KEY, 0u, 0u, 0u);
       if (valid) {
         uint32_t slot = fmix32(h.x) & (cap - 1);
-        for (;;) {
-          e = s_hash[slot];
-          if (e.x == h.x || e.x == EMPTY_KEY) break;
+        e = s_hash[slot];
+        while (e.x != h.x && e.x != EMPTY_KEY) {  // collision: linear probing (load <= 1/2, rare)
           slot = (slot + 1) & (cap - 1);
+          e = s_hash[slot];
         }
       }
       const bool known = valid && e.x == h.x && h.x != EMPTY_KEY;  // 0xFFFFFFFF is never registered
@@ -544,7 +563,11 @@ KernelFn select_kernel(uint32_t mask) {
 }  // namespace
 
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
-  size_t words = kSmVar + 4ull * c->cap + 4ull * c->nvd + (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
+  const uint32_t H = c->mask;
+  size_t words = sm_var_words(H) + 4ull * c->cap;
+  if (H & SASSI_H_VALUE) words += 4ull * c->nvd;
+  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
+    words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
   *bytes = 4 * words;
   return 0;
 }
