@@ -26,13 +26,12 @@ constexpr uint32_t I_ELIGIBLE = 1u << 3;      // instcount-eligible (R12)
 constexpr uint32_t I_NDST_SHIFT = 4;          // 3 bits: n_gpr_dst
 constexpr uint32_t I_VD0_SHIFT = 8;           // 16 bits: first value-destination state slot
 
-__host__ __device__ __forceinline__ uint32_t fmix32(uint32_t h) {
-  h ^= h >> 16;
-  h *= 0x85EBCA6Bu;
-  h ^= h >> 13;
-  h *= 0xC2B2AE35u;
-  h ^= h >> 16;
-  return h;
+// Home slot of a pc in the site hash: multiplicative hash ((pc * mul) >> shr) & (cap - 1), its
+// parameters chosen per site table at attach time (capi.cu choose_hash): for the dense pcs of a
+// real kernel (one SASS instruction every 16 B) mul = 1, shr = 4 is collision-free.
+__host__ __device__ __forceinline__ uint32_t pc_slot(uint32_t pc, uint32_t mul, uint32_t shr,
+                                                     uint32_t cap) {
+  return ((pc * mul) >> shr) & (cap - 1);
 }
 
 // Table image offsets (u64 words), same formulas as sassi_table_layout().
@@ -51,6 +50,7 @@ struct ConsumeParams {
   uint64_t arow_end, vrow_end;      // one past the last valid row index (bounds check)
   const uint4* hash;                // [cap] {key, info, cidx, 0}
   uint32_t cap;                     // power of two
+  uint32_t hmul, hshr;              // pc_slot parameters
   uint32_t nb, nm, nv, nvd;         // branch sites, memdiv sites, value sites, value (site,dst)s
   uint32_t pw;                      // private counter words per warp (16 B multiple)
   uint32_t priv;                    // 1: per-warp private counters; 0: one shared set + atomics
@@ -80,6 +80,7 @@ struct sassi_ctx {
   uint32_t cap_base = 0;            // pow2 >= 2 * n_sites
   uint32_t hash_cap = 0;            // capacity of the table on the device
   uint32_t cap = 0;
+  uint32_t hmul = 1, hshr = 4;      // pc_slot parameters of the table on the device
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
   uint32_t* d_err = nullptr;

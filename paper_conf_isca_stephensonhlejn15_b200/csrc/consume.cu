@@ -67,8 +67,9 @@ __device__ __forceinline__ T warp_sort(T v, uint32_t lane) {
 
 // Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
 // over the lanes of G (the count of Fig.6's leader-election loop, l.16-26).
-//  - window path: every sector within [-32, 31] of the first G lane's (same high word): a 64-bit
-//    window bitmap OR-reduced across the warp (REDUX), popcount.
+//  - window path: every sector of G within the 32-sector (1 KB, 8-line) window that starts at the
+//    line holding the lowest sector (same high word): the window bitmap is OR-reduced across the
+//    warp (REDUX), s = its popcount, L = the popcount of its nibbles OR-folded (a nibble = a line).
 //  - otherwise: sort the keys across the warp (bitonic, 32-bit when all high words agree) with the
 //    lanes outside G padded to the maximum so they sort last, and count positions < n whose key
 //    differs from the previous one; lines come from the same sorted sectors (>> 2 keeps order).
@@ -77,16 +78,14 @@ __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane
   const bool in = (G >> lane) & 1u;
   const uint64_t sec = a >> 5;
   const uint32_t slo = (uint32_t)sec, shi = (uint32_t)(sec >> 32);
-  const int leader = __ffs(G) - 1;
-  const uint32_t blo = __shfl_sync(FULL, slo, leader), bhi = __shfl_sync(FULL, shi, leader);
-  const uint32_t e = slo - blo + 32u;  // window position, valid when < 64 and high words agree
+  const uint32_t bhi = __reduce_max_sync(FULL, in ? shi : 0u);
+  const uint32_t base = __reduce_min_sync(FULL, in ? slo : FULL) & ~3u;  // line-aligned
+  const uint32_t e = slo - base;  // window position, valid when < 32 and high words agree
   const bool same_hi = !in || shi == bhi;
-  if (__all_sync(FULL, same_hi && (!in || e < 64u))) {
-    const uint32_t lo = __reduce_or_sync(FULL, in ? (1u << e) : 0u);          // e >= 32 -> 0
-    const uint32_t hi = __reduce_or_sync(FULL, in ? (1u << (e - 32u)) : 0u);  // e < 32 -> 0
-    const uint32_t ln = (uint32_t)(((int32_t)(e - 32u) + (int32_t)(blo & 3u)) >> 2) + 8u;  // 0..16
-    *out_s = __popc(lo) + __popc(hi);
-    *out_l = __popc(__reduce_or_sync(FULL, in ? (1u << ln) : 0u));
+  if (__all_sync(FULL, same_hi && (!in || e < 32u))) {
+    const uint32_t m = __reduce_or_sync(FULL, in ? (1u << e) : 0u);
+    *out_s = __popc(m);
+    *out_l = __popc((m | (m >> 1) | (m >> 2) | (m >> 3)) & 0x11111111u);
     return;
   }
   const uint32_t n = __popc(G);
@@ -269,7 +268,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239) ----
       uint4 e = make_uint4(EMPTY_KEY, 0u, 0u, 0u);
       if (valid) {
-        uint32_t slot = fmix32(h.x) & (cap - 1);
+        uint32_t slot = pc_slot(h.x, p.hmul, p.hshr, cap);
         e = s_hash[slot];
         while (e.x != h.x && e.x != EMPTY_KEY) {  // collision: linear probing (load <= 1/2, rare)
           slot = (slot + 1) & (cap - 1);

@@ -9,7 +9,8 @@ namespace {
 // one warp per chunk: per-chunk addr-row and val-row counts
 __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restrict__ hdr, uint64_t n,
                                                            const uint4* __restrict__ hash,
-                                                           uint32_t cap, uint64_t* na, uint64_t* nv) {
+                                                           uint32_t cap, uint32_t hmul, uint32_t hshr,
+                                                           uint64_t* na, uint64_t* nv) {
   const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t nch = (n + SASSI_CHUNK - 1) / SASSI_CHUNK;
@@ -19,7 +20,7 @@ __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restri
     const uint64_t i = c * SASSI_CHUNK + k;
     if (i >= n) break;
     const uint32_t pc = hdr[i].x;
-    uint32_t slot = fmix32(pc) & (cap - 1);
+    uint32_t slot = pc_slot(pc, hmul, hshr, cap);
     for (;;) {
       const uint4 e = hash[slot];
       const uint32_t key = e.x;
@@ -59,7 +60,7 @@ int launch_index(sassi_ctx* c, const sassi_hdr* hdr, uint64_t n, sassi_chunk_bas
   uint64_t *na = buf, *nv = buf + nch, *Pa = nv + nch, *Pv = Pa + nch + 1, *scratch = Pv + nch + 1;
   if (nch) {
     chunk_counts_kernel<<<(unsigned)((nch * 32 + 255) / 256), 256, 0, s>>>(
-        reinterpret_cast<const uint4*>(hdr), n, c->d_hash, c->cap, na, nv);
+        reinterpret_cast<const uint4*>(hdr), n, c->d_hash, c->cap, c->hmul, c->hshr, na, nv);
     SASSI_CUDA(cudaGetLastError());
   }
   int rc = scan_u64(na, nch, Pa, scratch, s);
