@@ -65,16 +65,30 @@ __device__ __forceinline__ T warp_sort(T v, uint32_t lane) {
   return v;
 }
 
+// {distinct sectors, distinct lines} of one row from its sorted sector keys (lanes outside G sort
+// last): the positions < n whose key differs from the previous one.
+template <typename T>
+__device__ __forceinline__ void count_sorted(T v, uint32_t n, uint32_t lane, uint32_t* out_s,
+                                             uint32_t* out_l) {
+  const T pv = __shfl_up_sync(FULL, v, 1);
+  const bool new_s = lane < n && (lane == 0 || v != pv);
+  const bool new_l = lane < n && (lane == 0 || (v >> 2) != (pv >> 2));
+  *out_s = __popc(__ballot_sync(FULL, new_s));
+  *out_l = __popc(__ballot_sync(FULL, new_l));
+}
+
 // Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
 // over the lanes of G (the count of Fig.6's leader-election loop, l.16-26).
 //  - window path: every sector of G within the 32-sector (1 KB, 8-line) window that starts at the
 //    line holding the lowest sector (same high word): the window bitmap is OR-reduced across the
 //    warp (REDUX), s = its popcount, L = the popcount of its nibbles OR-folded (a nibble = a line).
-//  - otherwise: sort the keys across the warp (bitonic, 32-bit when all high words agree) with the
+//  - otherwise, when all high words agree: sort the 32-bit keys across the warp (bitonic) with the
 //    lanes outside G padded to the maximum so they sort last, and count positions < n whose key
 //    differs from the previous one; lines come from the same sorted sectors (>> 2 keeps order).
-__device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
-                                           uint32_t* out_l) {
+//  - rows whose sectors differ in the high word return false and go to memdiv_row64 (64-bit keys),
+//    called once per such row outside the unrolled row loop to keep that loop's code small.
+__device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
+                                             uint32_t* out_l) {
   const bool in = (G >> lane) & 1u;
   const uint64_t sec = a >> 5;
   const uint32_t slo = (uint32_t)sec, shi = (uint32_t)(sec >> 32);
@@ -86,23 +100,17 @@ __device__ __forceinline__ void memdiv_row(uint64_t a, uint32_t G, uint32_t lane
     const uint32_t m = __reduce_or_sync(FULL, in ? (1u << e) : 0u);
     *out_s = __popc(m);
     *out_l = __popc((m | (m >> 1) | (m >> 2) | (m >> 3)) & 0x11111111u);
-    return;
+    return true;
   }
-  const uint32_t n = __popc(G);
-  bool new_s, new_l;
-  if (__all_sync(FULL, same_hi)) {
-    const uint32_t v = warp_sort<uint32_t>(in ? slo : FULL, lane);
-    const uint32_t pv = __shfl_up_sync(FULL, v, 1);
-    new_s = lane < n && (lane == 0 || v != pv);
-    new_l = lane < n && (lane == 0 || (v >> 2) != (pv >> 2));
-  } else {
-    const uint64_t v = warp_sort<uint64_t>(in ? sec : ~0ull, lane);
-    const uint64_t pv = __shfl_up_sync(FULL, v, 1);
-    new_s = lane < n && (lane == 0 || v != pv);
-    new_l = lane < n && (lane == 0 || (v >> 2) != (pv >> 2));
-  }
-  *out_s = __popc(__ballot_sync(FULL, new_s));
-  *out_l = __popc(__ballot_sync(FULL, new_l));
+  if (!__all_sync(FULL, same_hi)) return false;
+  count_sorted(warp_sort<uint32_t>(in ? slo : FULL, lane), __popc(G), lane, out_s, out_l);
+  return true;
+}
+
+__device__ __forceinline__ void memdiv_row64(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
+                                             uint32_t* out_l) {
+  const bool in = (G >> lane) & 1u;
+  count_sorted(warp_sort<uint64_t>(in ? (a >> 5) : ~0ull, lane), __popc(G), lane, out_s, out_l);
 }
 
 // ---- TMA bulk copy global -> shared with an mbarrier (cp.async.bulk, SASS UBLKCP) ----
@@ -350,6 +358,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
           const uint64_t* const abase = achunk + 32 * arow_b + lane;
           const uint32_t arel = __popc(ma & lt);
           uint32_t my_s = 0, my_l = 0;  // results of this lane's own record
+          uint32_t slow = 0;            // rows whose sectors differ in the high word
           do {
             uint64_t a[4];
             uint32_t g[4], jj[4];
@@ -368,14 +377,28 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
             for (int k = 0; k < 4; ++k) {
               if (g[k]) {
                 uint32_t s, L;
-                memdiv_row(a[k], g[k], lane, &s, &L);
-                if (lane == jj[k]) {
-                  my_s = s;
-                  my_l = L;
+                if (memdiv_row32(a[k], g[k], lane, &s, &L)) {
+                  if (lane == jj[k]) {
+                    my_s = s;
+                    my_l = L;
+                  }
+                } else {
+                  slow |= 1u << jj[k];
                 }
               }
             }
           } while (selm);
+          while (slow) {
+            const int j = __ffs(slow) - 1;
+            slow &= slow - 1;
+            uint32_t s, L;
+            memdiv_row64(ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j)), __shfl_sync(FULL, G, j),
+                         lane, &s, &L);
+            if (lane == j) {
+              my_s = s;
+              my_l = L;
+            }
+          }
           // one vectorised update for the batch: each record's lane adds its own results
           const uint32_t n = __popc(G);
           if (selm_l) {

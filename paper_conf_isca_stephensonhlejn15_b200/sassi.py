@@ -12,7 +12,8 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libsassi.so")
+# SASSI_LIB selects another build of the same library (tools/build_variant.py A/B timing)
+LIB_PATH = os.environ.get("SASSI_LIB") or os.path.join(_PKG, "lib", "libsassi.so")
 
 SITE_DTYPE = np.dtype([("pc", "<u4"), ("flags", "<u2"), ("mem_width", "u1"), ("domain", "u1"),
                        ("n_gpr_dst", "u1"), ("reg_num", "u1", (4,)), ("reserved", "u1", (3,))])
