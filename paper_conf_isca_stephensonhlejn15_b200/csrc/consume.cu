@@ -144,15 +144,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   }
 }
 
-// Per-record counter update into the warp's private counter words: lanes whose records hit the
-// same site in this batch (short loop bodies) are detected with MATCH.ANY and fall back to
-// shared-memory atomics; all other lanes do a plain vector read-modify-write.
+// Per-record counter update into the warp's private counter words: a plain vector
+// read-modify-write, or shared-memory atomics for lanes flagged `dup` (their record's site also
+// occurs at another lane of the batch — short loop bodies — or the counters are not private).
 __device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, uint32_t* region,
-                                              uint32_t priv, uint32_t lane) {
-  const uint32_t part = __ballot_sync(FULL, pred);
-  if (part == 0) return;
-  bool dup = !priv;
-  if (priv && pred) dup = __match_any_sync(part, off) != (1u << lane);
+                                              bool dup) {
   if (pred && !dup) {
     uint4* q = reinterpret_cast<uint4*>(region + off);
     uint4 c = *q;
@@ -170,11 +166,7 @@ __device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, 
 }
 
 __device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, uint32_t* region,
-                                              uint32_t priv, uint32_t lane) {
-  const uint32_t part = __ballot_sync(FULL, pred);
-  if (part == 0) return;
-  bool dup = !priv;
-  if (priv && pred) dup = __match_any_sync(part, off) != (1u << lane);
+                                              bool dup) {
   if (pred && !dup) {
     uint2* q = reinterpret_cast<uint2*>(region + off);
     uint2 c = *q;
@@ -314,6 +306,11 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       const bool live = known && act != 0;
       c_inv += known && act == 0;
       const uint32_t G = act & h.w;  // guard-true (or taken) active lanes
+      // records of this batch that share their pc with another lane's (one MATCH.ANY per batch for
+      // every handler's counter update; padding lanes repeat the last pc, which is only slower)
+      bool dup = true;
+      if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
+        dup = !p.priv || __match_any_sync(FULL, h.x) != (1u << lane);
       // value rows of this batch are contiguous: start the first bulk copy now, so it lands while
       // the other handlers work on the batch
       const uint32_t* const vsrc = vchunk + 32 * vrow_b;
@@ -325,7 +322,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
         add_counters4(isb, 4 * (cidx & 0xFFFFu),
                       make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
                                  (G != 0 && G != act) ? 1u : 0u),
-                      wpriv, p.priv, lane);
+                      wpriv, dup);
       }
       // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
       if (H & SASSI_H_INSTCOUNT) {
@@ -406,14 +403,14 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
             atomicAdd(sm + kSmH128 + 32 * (n - 1) + (my_l - 1), 1u);
           }
           add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv,
-                        p.priv, lane);
+                        dup);
         }
       }
       // ---- Case study III: value profiling (Fig.9): row-per-lane fold of TMA-staged rows ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
         add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
-                      p.priv, lane);
+                      dup);
         if (vtot) {
           const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
           const uint32_t vslot = info >> I_VD0_SHIFT;         // its first value-state slot
