@@ -11,6 +11,10 @@
  *     - SASSI_H_VALUE     value profiling: constant bits + scalar writes (§7, Fig.9)
  *     - SASSI_H_INSTCOUNT per-thread dynamic-instruction counts for error-injection
  *                         site selection (§8.1)
+ *   plus the paper's introductory example handler:
+ *     - SASSI_H_INSTMIX   instruction mix: thread-level counts of memory / extended memory /
+ *                         control-transfer / sync / numeric / texture / all instructions
+ *                         (Fig.3)
  *   The handler semantics (which lanes count, init values, counter widths) are spelled out in
  *   DESIGN.md §3 ("Readings"); every table entry is an integer fold, so results are exact.
  *
@@ -60,6 +64,9 @@
  *   h32[32][32]    sassi_counters[numActive-1][unique-1], unique = distinct 32 B sectors (Fig.6 l.33)
  *   h128[32][32]   the same matrix with 128 B lines
  *   counts[32*W]   per-thread eligible dynamic-instruction counts (§8.1 (4), L627)
+ *   mix[S]         thread executions per site: sum of popc(active) (Fig.3's count, per site)
+ *   imix[8]        Fig.3's dynamic_instr_counts[7] = {memory, extended memory (width > 4 B),
+ *                  controlxfer, sync, numeric, texture, total executed}, then one zero word
  *
  * ---------------------------------------------------------------------------------------------
  * CONVENTIONS
@@ -80,7 +87,7 @@
 extern "C" {
 #endif
 
-#define SASSI_ABI_VERSION 1u
+#define SASSI_ABI_VERSION 2u
 #define SASSI_WARP_SIZE 32u
 #define SASSI_CHUNK 256u           /* records per chunk_base entry */
 #define SASSI_MAX_SITES 4096u      /* registered sites per context */
@@ -103,7 +110,9 @@ enum {
   SASSI_H_MEMDIV = 2u,
   SASSI_H_VALUE = 4u,
   SASSI_H_INSTCOUNT = 8u,
-  SASSI_H_ALL = 15u
+  SASSI_H_ALL = 15u,       /* the paper's four case-study handlers (§5-§8)                      */
+  SASSI_H_INSTMIX = 16u,   /* Fig.3 instruction mix (L193-L199)                                 */
+  SASSI_H_EVERY = 31u      /* every handler kind                                                */
 };
 
 /* sassi_site.flags — static instruction properties (insEncoding / properties). */
@@ -159,7 +168,7 @@ typedef struct sassi_inj_site {
 } sassi_inj_site;      /* 32 B */
 
 typedef struct sassi_layout {
-  uint64_t diag, br, mem, val, ones, zeros, scalar, h32, h128, counts, total; /* in u64 words */
+  uint64_t diag, br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, total; /* u64 words */
 } sassi_layout;
 
 /* Offsets of the table image (host-only arithmetic; no device needed). */
@@ -173,7 +182,8 @@ int sassi_ctx_create(struct sassi_ctx** out, int device, const sassi_site* sites
                      uint32_t n_warps);
 void sassi_ctx_destroy(struct sassi_ctx* ctx);
 
-/* Select which handlers run (SASSI_H_* mask) — the paper's "what" (L181-L187). Allowed only
+/* Select which handlers run (non-empty subset of SASSI_H_EVERY) — the paper's "what"
+ * (L181-L187). Allowed only
  * before the first consume or right after sassi_reset. Errors: EINVAL, ESTATE, ENOSPC. */
 int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
 

@@ -34,6 +34,10 @@ F_COND_BRANCH, F_CTRL, F_MEM, F_MEM_READ, F_MEM_WRITE = 1, 2, 4, 8, 16
 F_ATOMIC, F_SYNC, F_NUMERIC, F_TEXTURE, F_WRITES_PRED, F_WRITES_CC = 32, 64, 128, 256, 512, 1024
 D_GLOBAL, D_SHARED, D_LOCAL, D_CONST, D_TEX = 0, 1, 2, 3, 4
 H_BRANCH, H_MEMDIV, H_VALUE, H_INSTCOUNT, H_ALL = 1, 2, 4, 8, 15
+H_INSTMIX = 16  # Fig.3 instruction-mix handler
+# Fig.3's dynamic_instr_counts[7] order (L193): imix[0..6]
+IMIX_NAMES = ("memory", "extended memory", "controlxfer", "sync", "numeric", "texture",
+              "total executed")
 
 
 def layout(n_sites: int, n_warps: int) -> dict:
@@ -48,7 +52,9 @@ def layout(n_sites: int, n_warps: int) -> dict:
     L["h32"] = L["scalar"] + 4 * S
     L["h128"] = L["h32"] + 1024
     L["counts"] = L["h128"] + 1024
-    L["total"] = L["counts"] + 32 * W
+    L["mix"] = L["counts"] + 32 * W
+    L["imix"] = L["mix"] + S
+    L["total"] = L["imix"] + 8
     return L
 
 
@@ -67,7 +73,9 @@ def sections(table: np.ndarray, n_sites: int, n_warps: int) -> dict:
         "scalar": t[L["scalar"]:L["h32"]].reshape(S, 4),
         "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
         "h128": t[L["h128"]:L["counts"]].reshape(32, 32),
-        "counts": t[L["counts"]:L["total"]],
+        "counts": t[L["counts"]:L["mix"]],
+        "mix": t[L["mix"]:L["imix"]],
+        "imix": t[L["imix"]:L["total"]],
     }
 
 

@@ -5,14 +5,13 @@ Each function restates a summary the paper prints (PAPER.md = /root/reference/PA
   - table1_percent      : Table 1 static/dynamic divergent-branch % (L255-L271, L281)
   - fig7_pmf            : Fig.7 PMF over unique 32 B lines, thread-weighted (L373)
   - table2_percent      : Table 2 constant-bit / scalar %, static and dynamic (L577-L593, L613)
-The product package has its own copy (paper_conf_isca_stephensonhlejn15_b200/reports.py); the two
-are compared in tests so neither is trusted alone.
+  - instmix_report      : Fig.3's dynamic_instr_counts[7] by category, with % of executed (L193-L199)
 """
 from __future__ import annotations
 
 import numpy as np
 
-from . import sections
+from . import IMIX_NAMES, sections
 
 
 def value_profile_lines(table, sites, n_warps):
@@ -87,3 +86,12 @@ def table2_percent(table, sites, n_warps):
     if n_s == 0:
         return 0.0, 0.0, 0.0, 0.0
     return 100 * cb_d / w_d, 100 * sc_d / w_d, 100 * cb_s / n_s, 100 * sc_s / n_s
+
+
+def instmix_report(table, n_sites, n_warps):
+    """Fig.3 (L193-L199): the seven thread-level counters [memory, extended memory, controlxfer,
+    sync, numeric, texture, total executed] as (name, count, % of total executed); categories
+    overlap, so the percentages need not sum to 100."""
+    imix = [int(x) for x in sections(table, n_sites, n_warps)["imix"][:7]]
+    tot = imix[6]
+    return [(n, c, 100.0 * c / tot if tot else 0.0) for n, c in zip(IMIX_NAMES, imix)]

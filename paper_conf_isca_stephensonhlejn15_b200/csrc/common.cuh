@@ -36,7 +36,7 @@ __host__ __device__ __forceinline__ uint32_t pc_slot(uint32_t pc, uint32_t mul, 
 
 // Table image offsets (u64 words), same formulas as sassi_table_layout().
 struct Offsets {
-  uint64_t br, mem, val, ones, zeros, scalar, h32, h128, counts, total;
+  uint64_t br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, total;
 };
 
 // Kernel parameter block of the fused consume kernel.
@@ -58,6 +58,9 @@ struct ConsumeParams {
   const uint32_t* flush_b;          // [nb] site index of branch compact slot
   const uint32_t* flush_m;          // [nm] site index of memdiv compact slot
   const uint32_t* flush_v;          // [nv][3] site index, first value-dst slot, n_dst
+  const uint32_t* flush_x;          // [S] Fig.3 category bits of each site (instruction mix)
+  uint32_t S;                       // registered sites
+  uint32_t px;                      // first private word of the per-site mix counters
   uint64_t* table;                  // device table image
   Offsets off;
   uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
@@ -82,6 +85,8 @@ struct sassi_ctx {
   uint32_t cap = 0;
   uint32_t hmul = 1, hshr = 4;      // pc_slot parameters of the table on the device
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
+  uint32_t pw_base = 0;             // private words of the branch / memdiv / value counters
+  std::vector<uint32_t> mix_cat;    // per site: Fig.3 category bits (bit c = dynamic_instr_counts[c])
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
   uint32_t* d_err = nullptr;
   uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums

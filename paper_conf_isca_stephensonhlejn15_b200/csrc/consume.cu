@@ -5,15 +5,19 @@
 // to the global u64 table image at CTA exit. Handlers (PAPER.md = /root/reference/PAPER.md):
 //   branch     Fig.4 (L237-L243)   lane-per-record: popc of active / taken masks
 //   memdiv     Fig.6 (L361-L369)   warp-per-row: distinct 32 B sectors and 128 B lines among the
-//                                  guard-true lanes; window-bitmap REDUX fast path, MATCH.ANY slow path
+//                                  guard-true lanes; window-bitmap REDUX fast path, warp sort otherwise
 //   value      Fig.9 (L549-L563)   row-per-lane: a batch's contiguous value rows are bulk-copied
 //                                  (TMA, cp.async.bulk + mbarrier) into the warp's shared-memory
 //                                  buffer; lane j folds row j's 32 values (AND / OR of the written
 //                                  lanes) -> constantOnes / constantZeros / isScalar
 //   instcount  §8.1 (L625-L627)    lane-per-record: 32x32 bit-matrix transpose + popc gives the
 //                                  per-lane count of 32 records; register accumulator per trace warp
+//   instmix    Fig.3 (L193-L199)   lane-per-record: popc(active) into a per-site counter; the seven
+//                                  category totals are formed at the flush
 // Work split: a warp owns one 256-record chunk at a time (chunk_base gives its row offsets) and walks
 // it in 8 batches of 32 records; row indices inside a batch come from ballot prefix sums.
+#include <utility>
+
 #include "common.cuh"
 
 namespace sassi {
@@ -144,20 +148,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   }
 }
 
-// Per-record counter update into the warp's private counter words: a plain vector
-// read-modify-write, or shared-memory atomics for lanes flagged `dup` (their record's site also
-// occurs at another lane of the batch — short loop bodies — or the counters are not private).
-__device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, uint32_t* region,
-                                              bool dup) {
-  if (pred && !dup) {
-    uint4* q = reinterpret_cast<uint4*>(region + off);
-    uint4 c = *q;
-    c.x += v.x;
-    c.y += v.y;
-    c.z += v.z;
-    c.w += v.w;
-    *q = c;
-  } else if (pred) {
+// Per-record counter update into the warp's private counter words: shared-memory atomics
+// (lanes whose records hit the same site in one batch — short loop bodies — add correctly, and
+// no duplicate detection is needed; a MATCH.ANY-guarded plain read-modify-write measured slower).
+__device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, uint32_t* region) {
+  if (pred) {
     atomicAdd(region + off, v.x);
     atomicAdd(region + off + 1, v.y);
     atomicAdd(region + off + 2, v.z);
@@ -165,15 +160,8 @@ __device__ __forceinline__ void add_counters4(bool pred, uint32_t off, uint4 v, 
   }
 }
 
-__device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, uint32_t* region,
-                                              bool dup) {
-  if (pred && !dup) {
-    uint2* q = reinterpret_cast<uint2*>(region + off);
-    uint2 c = *q;
-    c.x += v.x;
-    c.y += v.y;
-    *q = c;
-  } else if (pred) {
+__device__ __forceinline__ void add_counters2(bool pred, uint32_t off, uint2 v, uint32_t* region) {
+  if (pred) {
     atomicAdd(region + off, v.x);
     atomicAdd(region + off + 1, v.y);
   }
@@ -186,9 +174,10 @@ template <uint32_t H>
 struct SmLayout {
   static constexpr bool kMem = (H & SASSI_H_MEMDIV) != 0, kVal = (H & SASSI_H_VALUE) != 0;
   static constexpr uint32_t kDiag = 0;                                  // 8 u32
-  static constexpr uint32_t kH32 = 8;                                   // [32][32] u32 (memdiv)
+  static constexpr uint32_t kImix = 8;                                  // 8 u64 (instmix totals)
+  static constexpr uint32_t kH32 = 24;                                  // [32][32] u32 (memdiv)
   static constexpr uint32_t kH128 = kH32 + 1024;                        // [32][32] u32 (memdiv)
-  static constexpr uint32_t kBar = kMem ? kH128 + 1024 : 8;             // [warps] u64 (value)
+  static constexpr uint32_t kBar = kMem ? kH128 + 1024 : 24;            // [warps] u64 (value)
   static constexpr uint32_t kVbuf = kVal ? ((kBar + 2 * kWarpsPerCta + 31) & ~31u) : kBar;
   static constexpr uint32_t kVar = kVbuf + (kVal ? kWarpsPerCta * kVbufWords : 0u);  // hash, ...
   static_assert(kVbuf % 32 == 0 || !kVal, "value buffers must be 128 B aligned");
@@ -197,7 +186,7 @@ struct SmLayout {
 // host mirror of SmLayout<H>::kVar
 uint32_t sm_var_words(uint32_t H) {
   const bool mem = H & SASSI_H_MEMDIV, val = H & SASSI_H_VALUE;
-  const uint32_t bar = mem ? 8 + 2048 : 8;
+  const uint32_t bar = mem ? 24 + 2048 : 24;
   const uint32_t vbuf = val ? ((bar + 2 * kWarpsPerCta + 31) & ~31u) : bar;
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
 }
@@ -206,8 +195,9 @@ template <uint32_t H>
 __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
   using Ly = SmLayout<H>;
-  constexpr uint32_t kSmDiag = Ly::kDiag, kSmH32 = Ly::kH32, kSmH128 = Ly::kH128, kSmBar = Ly::kBar,
-                     kSmVbuf = Ly::kVbuf, kSmVar = Ly::kVar;
+  constexpr uint32_t kSmDiag = Ly::kDiag, kSmImix = Ly::kImix, kSmH32 = Ly::kH32, kSmH128 = Ly::kH128,
+                     kSmBar = Ly::kBar, kSmVbuf = Ly::kVbuf, kSmVar = Ly::kVar;
+  constexpr uint32_t kCounters = SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX;
   const uint32_t cap = p.cap;
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
   uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
@@ -218,7 +208,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
   for (uint32_t i = tid; i < cap; i += blockDim.x) s_hash[i] = p.hash[i];
   if (Ly::kVal)
     for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
-  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
+  if (H & kCounters)
     for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
   for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
   if (Ly::kVal && tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
@@ -306,11 +296,6 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       const bool live = known && act != 0;
       c_inv += known && act == 0;
       const uint32_t G = act & h.w;  // guard-true (or taken) active lanes
-      // records of this batch that share their pc with another lane's (one MATCH.ANY per batch for
-      // every handler's counter update; padding lanes repeat the last pc, which is only slower)
-      bool dup = true;
-      if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
-        dup = !p.priv || __match_any_sync(FULL, h.x) != (1u << lane);
       // value rows of this batch are contiguous: start the first bulk copy now, so it lands while
       // the other handlers work on the batch
       const uint32_t* const vsrc = vchunk + 32 * vrow_b;
@@ -322,8 +307,11 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
         add_counters4(isb, 4 * (cidx & 0xFFFFu),
                       make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
                                  (G != 0 && G != act) ? 1u : 0u),
-                      wpriv, dup);
+                      wpriv);
       }
+      // ---- Fig.3 instruction mix (L193-L199): every active thread counts; per-site thread
+      // executions here, the seven category totals at the flush (R22) ----
+      if ((H & SASSI_H_INSTMIX) && live) atomicAdd(wpriv + p.px + e.w, (uint32_t)__popc(act));
       // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
       if (H & SASSI_H_INSTCOUNT) {
         uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
@@ -402,15 +390,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
             atomicAdd(sm + kSmH32 + 32 * (n - 1) + (my_s - 1), 1u);
             atomicAdd(sm + kSmH128 + 32 * (n - 1) + (my_l - 1), 1u);
           }
-          add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv,
-                        dup);
+          add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv);
         }
       }
       // ---- Case study III: value profiling (Fig.9): row-per-lane fold of TMA-staged rows ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
-        add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv,
-                      dup);
+        add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv);
         if (vtot) {
           const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
           const uint32_t vslot = info >> I_VD0_SHIFT;         // its first value-state slot
@@ -530,6 +516,20 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       if (v) atomicAdd(table + (c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024)), (unsigned long long)v);
     }
   }
+  if (H & SASSI_H_INSTMIX) {
+    unsigned long long* const s_imix = reinterpret_cast<unsigned long long*>(sm + kSmImix);
+    for (uint32_t st = tid; st < p.S; st += blockDim.x) {
+      uint32_t t = 0;
+      for (uint32_t w = 0; w < n_regions; ++w) t += s_priv[w * p.pw + p.px + st];
+      if (t == 0) continue;
+      atomicAdd(table + p.off.mix + st, (unsigned long long)t);
+      const uint32_t cat = p.flush_x[st];
+      for (uint32_t k = 0; k < 7; ++k)
+        if ((cat >> k) & 1u) atomicAdd(s_imix + k, (unsigned long long)t);
+    }
+    __syncthreads();
+    if (tid < 7 && s_imix[tid]) atomicAdd(table + p.off.imix + tid, s_imix[tid]);
+  }
   if (H & SASSI_H_VALUE) {
     for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
       const uint32_t site = p.flush_v[3 * k], vd0 = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
@@ -558,25 +558,17 @@ KernelFn kernel_for() {
   return consume_kernel<H>;
 }
 
+template <uint32_t... Hs>
+KernelFn pick(uint32_t mask, std::integer_sequence<uint32_t, Hs...>) {
+  KernelFn fn = nullptr;
+  ((mask == Hs + 1 ? (fn = kernel_for<Hs + 1>(), 0) : 0), ...);
+  return fn;
+}
+
+// one instantiation per non-empty handler set (1..31)
 KernelFn select_kernel(uint32_t mask) {
-  switch (mask & 15u) {
-    case 1: return kernel_for<1>();
-    case 2: return kernel_for<2>();
-    case 3: return kernel_for<3>();
-    case 4: return kernel_for<4>();
-    case 5: return kernel_for<5>();
-    case 6: return kernel_for<6>();
-    case 7: return kernel_for<7>();
-    case 8: return kernel_for<8>();
-    case 9: return kernel_for<9>();
-    case 10: return kernel_for<10>();
-    case 11: return kernel_for<11>();
-    case 12: return kernel_for<12>();
-    case 13: return kernel_for<13>();
-    case 14: return kernel_for<14>();
-    case 15: return kernel_for<15>();
-    default: return nullptr;
-  }
+  if (mask == 0 || mask > SASSI_H_EVERY) return nullptr;
+  return pick(mask, std::make_integer_sequence<uint32_t, SASSI_H_EVERY>{});
 }
 
 }  // namespace
@@ -585,7 +577,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   const uint32_t H = c->mask;
   size_t words = sm_var_words(H) + 4ull * c->cap;
   if (H & SASSI_H_VALUE) words += 4ull * c->nvd;
-  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE))
+  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX))
     words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
   *bytes = 4 * words;
   return 0;

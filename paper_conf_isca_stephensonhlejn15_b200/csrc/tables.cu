@@ -14,7 +14,9 @@ Offsets layout_offsets(uint32_t S, uint32_t W) {
   o.h32 = o.scalar + 4ull * S;
   o.h128 = o.h32 + 1024;
   o.counts = o.h128 + 1024;
-  o.total = o.counts + 32ull * W;
+  o.mix = o.counts + 32ull * W;
+  o.imix = o.mix + S;
+  o.total = o.imix + 8;
   return o;
 }
 
@@ -63,6 +65,8 @@ extern "C" int sassi_table_layout(uint32_t n_sites, uint32_t n_warps, sassi_layo
   out->h32 = o.h32;
   out->h128 = o.h128;
   out->counts = o.counts;
+  out->mix = o.mix;
+  out->imix = o.imix;
   out->total = o.total;
   return SASSI_OK;
 }

@@ -24,6 +24,7 @@ INJ_DTYPE = np.dtype([("kernel", "<u4"), ("invocation", "<u4"), ("thread", "<u4"
 SASSI_OK, SASSI_EINVAL, SASSI_ECUDA, SASSI_ENCCL = 0, -1, -2, -3
 SASSI_ENOSPC, SASSI_ESTATE, SASSI_EMISMATCH, SASSI_EFORMAT = -4, -5, -6, -7
 SASSI_H_BRANCH, SASSI_H_MEMDIV, SASSI_H_VALUE, SASSI_H_INSTCOUNT, SASSI_H_ALL = 1, 2, 4, 8, 15
+SASSI_H_INSTMIX, SASSI_H_EVERY = 16, 31
 SASSI_CHUNK = 256
 SASSI_IK_VECADD, SASSI_IK_BFS, SASSI_IK_SGEMM, SASSI_IK_STENCIL = 0, 1, 2, 3
 SASSI_IK_NONE, SASSI_IK_TRACE, SASSI_IK_NULL_ABI = 0, 16, 32
@@ -39,7 +40,7 @@ class SassiRecords(ctypes.Structure):
 
 class SassiLayout(ctypes.Structure):
     _fields_ = [(k, _u64) for k in ("diag", "br", "mem", "val", "ones", "zeros", "scalar", "h32",
-                                    "h128", "counts", "total")]
+                                    "h128", "counts", "mix", "imix", "total")]
 
 
 SIGNATURES = {
@@ -260,7 +261,8 @@ class Context:
                 "zeros": t[L["zeros"]:L["scalar"]].reshape(S, 4),
                 "scalar": t[L["scalar"]:L["h32"]].reshape(S, 4),
                 "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
-                "h128": t[L["h128"]:L["counts"]].reshape(32, 32), "counts": t[L["counts"]:L["total"]]}
+                "h128": t[L["h128"]:L["counts"]].reshape(32, 32), "counts": t[L["counts"]:L["mix"]],
+                "mix": t[L["mix"]:L["imix"]], "imix": t[L["imix"]:L["total"]]}
 
     def sample(self, k: int, seed: int, stream=None) -> np.ndarray:
         return sassi_sample_sites(self.handle, k, seed, stream)

@@ -2,7 +2,8 @@
 
 Every expected number below was computed on paper from the handler listings, not by any code:
   Fig.4 (L237-L243) branch, Fig.6 (L361-L369) memory divergence, Fig.9 (L549-L563) value profile,
-  §8.1 (L625-L627) per-thread counts; readings R1-R13 of DESIGN.md §3.
+  §8.1 (L625-L627) per-thread counts, Fig.3 (L193-L199) instruction mix; readings R1-R13 and R22
+  of DESIGN.md §3.
 """
 import numpy as np
 
@@ -19,7 +20,7 @@ def sites():
     rows = [
         (0x10, F_COND_BRANCH | F_CTRL, 0, D_GLOBAL, 0, [0, 0, 0, 0]),             # s0 BRA
         (0x20, F_MEM | F_MEM_READ, 4, D_GLOBAL, 1, [12, 0, 0, 0]),               # s1 LDG R12
-        (0x30, F_MEM | F_MEM_WRITE, 4, D_GLOBAL, 0, [0, 0, 0, 0]),               # s2 STG
+        (0x30, F_MEM | F_MEM_WRITE, 8, D_GLOBAL, 0, [0, 0, 0, 0]),               # s2 STG.64
         (0x40, F_NUMERIC, 0, D_GLOBAL, 1, [13, 0, 0, 0]),                        # s3 IADD R13
         (0x50, F_MEM | F_MEM_READ, 4, D_SHARED, 1, [14, 0, 0, 0]),               # s4 LDS R14
         (0x60, F_NUMERIC | F_WRITES_PRED, 0, D_GLOBAL, 0, [0, 0, 0, 0]),         # s5 ISETP
@@ -117,6 +118,14 @@ def expect_counts():
     return c
 
 
+# Fig.3 (R22): every ACTIVE thread counts (guard-false lanes too), per site Σ popc(active):
+#   s0 32+32+16, s1 32+32+4+32, s2 32 (lane 5 guard-false still counts), s3 32+2 (+0 for r13),
+#   s4 32, s5 32, s6 32; r12 is unregistered.
+EXPECT_MIX = [80, 100, 32, 34, 32, 32, 32]
+# memory = s1+s2+s4 = 164; extended (width > 4) = s2 = 32; controlxfer = s0 = 80; sync = s6 = 32;
+# numeric = s3+s5 = 66; texture = 0; total = 342
+EXPECT_IMIX = [164, 32, 80, 32, 66, 0, 342, 0]
+
 EXPECT_VALUE_LINES = {
     0x20: ["R12 <- [000000000000000000000000000TTTTT]"],
     0x40: ["R13* <- [00000000000000000000000000000001]"],
@@ -124,8 +133,9 @@ EXPECT_VALUE_LINES = {
 }
 
 
-def check_table(t, sec):
-    """Assert a table image (dict of sections) equals the hand-worked expectation."""
+def check_table(t, sec, mask=15):
+    """Assert a table image (dict of sections) equals the hand-worked expectation (handlers 1-8
+    always; the Fig.3 sections when mask has 16, else they stay 0)."""
     assert list(map(int, sec["diag"][:4])) == EXPECT_DIAG
     S = 7
     for s in range(S):
@@ -147,3 +157,7 @@ def check_table(t, sec):
     assert np.array_equal(sec["h32"], h32)
     assert np.array_equal(sec["h128"], h128)
     assert np.array_equal(sec["counts"], expect_counts())
+    mix = EXPECT_MIX if mask & 16 else [0] * 7
+    imix = EXPECT_IMIX if mask & 16 else [0] * 8
+    assert list(map(int, sec["mix"])) == mix
+    assert list(map(int, sec["imix"])) == imix

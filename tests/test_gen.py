@@ -95,6 +95,26 @@ def test_c1_oracle_closed_forms():
     assert list(map(int, sec["diag"][:4])) == [4812, 0, 0, 0]
 
 
+def test_c1_instmix_closed_form():
+    """Fig.3 on c1 by hand: 128 threads; prologue 2 numeric; per iteration 6 numeric (2 IMAD.WIDE,
+    FADD, 2 ISETP, IADD), 3 memory (2 LDG, STG, all 4 B), 2 control transfers (2 BRA), and the
+    x[32 i] load on the 4,267 (thread, iteration) pairs with i % 3 == 0; EXIT is one more control
+    transfer per thread."""
+    P, lim, mask, _ = gen.preset("c1")
+    r = gen.generate_host(P, lim)
+    s = r["sites"]
+    t = oracle.run(s, 4, oracle.H_INSTMIX, r["hdr"], r["addr"], r["val"])
+    sec = oracle.sections(t, len(s), 4)
+    n3 = len(range(0, 12800, 3))
+    numeric = 2 * 128 + 6 * 12800
+    memory = 3 * 12800 + n3
+    ctrl = 2 * 12800 + 128
+    assert list(map(int, sec["imix"])) == [memory, 0, ctrl, 0, numeric, 0,
+                                           numeric + memory + ctrl, 0]
+    idx = {int(x["pc"]): i for i, x in enumerate(s)}
+    assert int(sec["mix"][idx[0x1A0]]) == n3 and int(sec["mix"][idx[0x140]]) == 12800
+
+
 def _walk_rows(sites, hdr):
     """(addr rows, val rows) before each record, from the site table only."""
     pcs = {int(x["pc"]): x for x in sites}

@@ -31,20 +31,23 @@ def test_t0_hand_worked_on_gpu():
     assert np.array_equal(t, oracle.run(s, T0.N_WARPS, oracle.H_ALL, hdr, addr, val))
 
 
-@pytest.mark.parametrize("mask", [1, 2, 4, 8, 3, 5, 6, 9, 10, 12, 7, 11, 13, 14, 15])
+@pytest.mark.parametrize("mask", list(range(1, 32)))
 def test_t0_every_handler_mask(mask):
     s = T0.sites()
     hdr, addr, val = T0.records()
     t = gpu_table(s, T0.N_WARPS, mask, to_device(s, hdr, addr, val))
     o = oracle.run(s, T0.N_WARPS, mask, hdr, addr, val)
     assert diff_tables(t, o, len(s), T0.N_WARPS) is None
+    if mask == sassi.SASSI_H_EVERY:       # every handler, hand-worked values included
+        T0.check_table(t, oracle.sections(t, len(s), T0.N_WARPS), mask)
 
 
 @pytest.mark.parametrize("seed,n", [(0, 1), (1, 31), (2, 257), (3, 1000), (4, 5000), (5, 20000)])
-def test_random_traces(seed, n):
+@pytest.mark.parametrize("mask", [sassi.SASSI_H_ALL, sassi.SASSI_H_EVERY, sassi.SASSI_H_INSTMIX])
+def test_random_traces(seed, n, mask):
     s, W, hdr, addr, val = random_trace(1000 + seed, n=n)
-    o = oracle.run(s, W, oracle.H_ALL, hdr, addr, val)
-    t = gpu_table(s, W, sassi.SASSI_H_ALL, to_device(s, hdr, addr, val))
+    o = oracle.run(s, W, mask, hdr, addr, val)
+    t = gpu_table(s, W, mask, to_device(s, hdr, addr, val))
     assert diff_tables(t, o, len(s), W) is None
 
 
@@ -108,17 +111,22 @@ def _gen(name, limit=None, warp_base=0, n_warps=None):
     return P, mask, gen.generate_device(P, lim, warp_base, n_warps)
 
 
-def test_c1_full():
+@pytest.mark.parametrize("every", [False, True])
+def test_c1_full(every):
     P, mask, d = _gen("c1")
+    mask = sassi.SASSI_H_EVERY if every else mask
     h = gen.to_host(d)
     t = gpu_table(h["sites"], P.total_warps, mask, d)
     o = oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"])
     assert diff_tables(t, o, len(h["sites"]), P.total_warps) is None
 
 
-def test_c2_full():
-    """Config 2 at its full size (10^7 records), bit-exact against the oracle."""
+@pytest.mark.parametrize("every", [False, True])
+def test_c2_full(every):
+    """Config 2 at its full size (10^7 records), bit-exact against the oracle (its four handlers,
+    and with the Fig.3 instruction mix added)."""
     P, mask, d = _gen("c2")
+    mask = sassi.SASSI_H_EVERY if every else mask
     assert d["n"] == 10_000_000
     h = gen.to_host(d)
     t = gpu_table(h["sites"], P.total_warps, mask, d)
