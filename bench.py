@@ -436,25 +436,26 @@ def main():
 def measure_slowdown(dev):
     """Instrumented-kernel slowdown K = t_instrumented / t_uninstrumented (the K column of the
     paper's Table 3), median of 5 runs each (L679), per handler, for the four synthetic
-    kernels at their timing sizes; `null_abi` is the paper's stubbed-handler control (L687)."""
+    kernels at their timing sizes; `null_abi` is the paper's stubbed-handler control (L687);
+    `instmix` is Fig.3's handler (L193-L199), `all` the four case studies, `every` all five."""
     import torch
     from paper_conf_isca_stephensonhlejn15_b200 import sassi
     modes = {"null_abi": sassi.SASSI_IK_NULL_ABI, "branch": 1, "memdiv": 2, "value": 4,
-             "instcount": 8, "all": 15}
+             "instcount": 8, "instmix": 16, "all": 15, "every": 31}
     out = {}
     stream = torch.cuda.current_stream(dev)
     for name in ("vecadd", "bfs", "sgemm", "stencil"):
         ik = sassi.InstrumentedKernel(name, 0, device=dev.index)
-        ctx = ik.context(sassi.SASSI_H_ALL)
+        ctx = ik.context(sassi.SASSI_H_EVERY)
 
         def timed(mode):
             ts = []
             for rep in range(6):
-                if mode & 15:
+                if mode & sassi.SASSI_H_EVERY:
                     ctx.reset(stream)
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record(stream)
-                ik.run(mode, ctx if mode & 15 else None, stream)
+                ik.run(mode, ctx if mode & sassi.SASSI_H_EVERY else None, stream)
                 b.record(stream)
                 b.synchronize()
                 if rep:

@@ -3,7 +3,9 @@
  *
  * Four CUDA kernels with hand-placed instrumentation sites, each runnable
  *   - uninstrumented (SASSI_IK_NONE) — the baseline t / k of Table 3;
- *   - with inline handlers (any SASSI_H_* mask) folding straight into a sassi_ctx's tables;
+ *   - with inline handlers folding straight into a sassi_ctx's tables: one handler
+ *     (SASSI_H_BRANCH / MEMDIV / VALUE / INSTCOUNT / INSTMIX), the four case studies
+ *     (SASSI_H_ALL) or every handler (SASSI_H_EVERY);
  *   - with a null handler called through a non-inlined ABI call with stack-allocated parameter
  *     objects (SASSI_IK_NULL_ABI) — the paper's stubbed-handler experiment (L687);
  *   - in trace mode (SASSI_IK_TRACE), appending SRF1 records per warp, so the same execution can
@@ -24,7 +26,7 @@ extern "C" {
 #endif
 
 enum { SASSI_IK_VECADD = 0, SASSI_IK_BFS = 1, SASSI_IK_SGEMM = 2, SASSI_IK_STENCIL = 3 };
-enum { SASSI_IK_NONE = 0u, SASSI_IK_TRACE = 16u, SASSI_IK_NULL_ABI = 32u };
+enum { SASSI_IK_NONE = 0u, SASSI_IK_TRACE = 64u, SASSI_IK_NULL_ABI = 128u };  /* above SASSI_H_EVERY */
 
 typedef struct sassi_ik sassi_ik;
 
@@ -36,7 +38,8 @@ void sassi_ik_destroy(sassi_ik* ik);
 /* The kernel's static site table (register it with sassi_ctx_create(sites, n_warps)). */
 int sassi_ik_sites(sassi_ik* ik, sassi_site* out, uint32_t cap, uint32_t* n_sites, uint32_t* n_warps);
 
-/* Run once. mode = SASSI_IK_NONE | SASSI_IK_NULL_ABI | SASSI_IK_TRACE | handler mask (SASSI_H_*);
+/* Run once. mode = SASSI_IK_NONE | SASSI_IK_NULL_ABI | SASSI_IK_TRACE | one of the handler masks
+ * above (1, 2, 4, 8, 16, 15, 31; EINVAL otherwise);
  * handler bits fold into ctx's tables (ctx must hold exactly this kernel's sites / warps).
  * Asynchronous on `stream` except SASSI_IK_TRACE, which synchronises. */
 int sassi_ik_run(sassi_ik* ik, uint32_t mode, struct sassi_ctx* ctx, void* stream);

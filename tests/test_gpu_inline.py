@@ -38,17 +38,18 @@ def trace_and_fold(ik, mask):
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-def test_inline_equals_trace_fold_equals_oracle(name):
+@pytest.mark.parametrize("mask", [sassi.SASSI_H_ALL, sassi.SASSI_H_EVERY])
+def test_inline_equals_trace_fold_equals_oracle(name, mask):
     ik = sassi.InstrumentedKernel(name, SMALL[name])
     S, W = len(ik.sites), ik.n_warps
-    ctx = ik.context(sassi.SASSI_H_ALL)
-    ik.run(sassi.SASSI_H_ALL, ctx)
+    ctx = ik.context(mask)
+    ik.run(mask, ctx)
     t_inline = ctx.read_tables()
     ctx.close()
-    rec, t_fold = trace_and_fold(ik, sassi.SASSI_H_ALL)
+    rec, t_fold = trace_and_fold(ik, mask)
     assert rec["n"] > 0
     h = gen.to_host(rec)
-    t_or = oracle.run(h["sites"], W, oracle.H_ALL, h["hdr"], h["addr"], h["val"])
+    t_or = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
     assert diff_tables(t_fold, t_or, S, W) is None
     assert int(t_inline[0]) == 0
     assert diff_tables(t_inline, no_diag(t_or), S, W) is None
@@ -56,7 +57,7 @@ def test_inline_equals_trace_fold_equals_oracle(name):
 
 
 @pytest.mark.parametrize("name", list(SMALL))
-@pytest.mark.parametrize("mask", [1, 2, 4, 8])
+@pytest.mark.parametrize("mask", [1, 2, 4, 8, 16])
 def test_single_handler_inline(name, mask):
     ik = sassi.InstrumentedKernel(name, SMALL[name])
     ctx = ik.context(mask)
@@ -74,12 +75,11 @@ def test_instrumentation_preserves_output(name):
     ik.run(sassi.SASSI_IK_NONE)
     torch.cuda.synchronize()
     base = ik.checksum()
-    ctx = ik.context(sassi.SASSI_H_ALL)
-    for mode in (sassi.SASSI_IK_NULL_ABI, sassi.SASSI_H_ALL, 1, 2, 4, 8):
-        ik.run(mode, ctx if mode & 15 else None)
+    ctx = ik.context(sassi.SASSI_H_EVERY)
+    for mode in (sassi.SASSI_IK_NULL_ABI, sassi.SASSI_H_ALL, 1, 2, 4, 8, 16, sassi.SASSI_H_EVERY):
+        ik.run(mode, ctx if mode & sassi.SASSI_H_EVERY else None)
         torch.cuda.synchronize()
         assert ik.checksum() == base, mode
-    ik.context(sassi.SASSI_H_ALL)
     ik.trace(ctx)
     assert ik.checksum() == base
     ctx.close()
