@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-slowdown", action="store_true")
+    ap.add_argument("--no-injection", action="store_true")
     return ap.parse_args()
 
 
@@ -390,6 +391,9 @@ def main():
     slow = None
     if not args.no_slowdown and rank == 0:
         slow = measure_slowdown(dev)
+    inj = None
+    if not args.no_injection and rank == 0:
+        inj = measure_injection(dev)
 
     if rank == 0:
         line = {
@@ -425,12 +429,39 @@ def main():
             line["cpu_baseline"] = cpu
         if slow:
             line["instrumented_slowdown"] = slow
+        if inj:
+            line["error_injection"] = inj
         print(json.dumps(line), flush=True)
     if comm is not None:
         sassi.sassi_nccl_comm_destroy(comm)
     ctx.close()
     if launched:
         dist.destroy_process_group()
+
+
+def measure_injection(dev, k=1000):
+    """§8.1's error-injection study on the four instrumented kernels (the Fig.10 analogue,
+    L637-L667): profile, draw k sites (L629), one run per site; % of runs per outcome and the
+    campaign's rate (runs/s, wall clock around the k runs: each run synchronises)."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    out = {}
+    for name in ("vecadd", "bfs", "sgemm", "stencil"):
+        ik = sassi.InstrumentedKernel(name, 0, device=dev.index)
+        ctx = ik.context(sassi.SASSI_H_INSTCOUNT)
+        ik.run(sassi.SASSI_H_INSTCOUNT, ctx)
+        sites = ctx.sample(k, 20150616)
+        ctx.close()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        outs = ik.inject(sites)
+        dt = time.perf_counter() - t0
+        r = {"runs": k, "runs_per_s": k / dt}
+        for code, nm in enumerate(sassi.INJ_OUTCOME_NAMES):
+            r[nm + "_pct"] = 100.0 * float((outs["outcome"] == code).sum()) / k
+        out[name] = r
+        ik.close()
+    return out
 
 
 def measure_slowdown(dev):

@@ -51,8 +51,36 @@ int sassi_ik_run(sassi_ik* ik, uint32_t mode, struct sassi_ctx* ctx, void* strea
 int sassi_ik_trace_totals(sassi_ik* ik, uint64_t* n_rec, uint64_t* n_addr_rows, uint64_t* n_val_rows);
 int sassi_ik_trace_copy(sassi_ik* ik, sassi_hdr* hdr, uint64_t* addr, uint32_t* val, void* stream);
 
-/* Checksum of the kernel's output buffer (to prove instrumentation does not change results). */
+/* Checksum of the kernel's output buffers (to prove instrumentation does not change results). */
 int sassi_ik_output_checksum(sassi_ik* ik, uint64_t* out);
+
+/* ---- Error injection (§8.1 step 3, L631-L633) -------------------------------
+ * One run per tuple (tuples as sassi_sample_sites draws them from a SASSI_H_INSTCOUNT profile of
+ * the same kernel): the thread `thread` counts its eligible, not-predicated-out dynamic
+ * instructions (the ones the profile counted, L627) and at number `dyn_index` (0-based) flips bit
+ * bit_seed % 32 of the value its destination register receives — the kernel continues with the
+ * corrupted value — or, for a store, of the 32-bit word it wrote (reading R23). The run
+ * is classified against an error-free reference run (L633):
+ *   MASKED       outputs identical
+ *   SDC          outputs differ (potential silent data corruption)
+ *   DUE          a corrupted data-dependent index left its array (the crash analogue: the
+ *                kernel checks the index, records the symptom and skips the access)
+ *   HANG         a loop ran past its watchdog (kHangCap trips)
+ *   NOT_REACHED  the thread executed fewer eligible instructions (outputs unchanged)
+ * Synchronises `stream` after every run; leaves the outputs as an error-free run leaves them. */
+enum { SASSI_INJ_MASKED = 0, SASSI_INJ_SDC = 1, SASSI_INJ_DUE = 2, SASSI_INJ_HANG = 3,
+       SASSI_INJ_NOT_REACHED = 4 };
+enum { SASSI_INJ_TARGET_GPR = 0, SASSI_INJ_TARGET_MEM = 1 };
+typedef struct sassi_ik_outcome {
+  uint32_t outcome;         /* SASSI_INJ_*                                                      */
+  uint32_t site;            /* static site of the injected instruction (0xFFFFFFFF: not reached) */
+  uint32_t target;          /* SASSI_INJ_TARGET_*                                               */
+  uint32_t bit;             /* flipped bit                                                      */
+  uint32_t before, after;   /* the value (GPR) or stored word (MEM) before / after the flip     */
+  uint32_t reserved[2];
+} sassi_ik_outcome;         /* 32 B */
+int sassi_ik_inject(sassi_ik* ik, const sassi_inj_site* sites, uint32_t n, sassi_ik_outcome* out,
+                    void* stream);
 
 #ifdef __cplusplus
 }

@@ -110,6 +110,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_sample.restype = ctypes.c_int
         L.oracle_splitmix64.argtypes = [u64]
         L.oracle_splitmix64.restype = u64
+        L.oracle_locate_injection.argtypes = [vp, u32, vp, u64, vp, u64, u64, u32, u32, vp]
+        L.oracle_locate_injection.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -168,3 +170,21 @@ def sample(counts: np.ndarray, k: int, seed: int) -> np.ndarray:
 
 def splitmix64(x: int) -> int:
     return int(lib().oracle_splitmix64(x & (2**64 - 1)))
+
+
+def locate_injection(sites, hdr, val, thread: int, dyn_index: int, reg_seed: int, bit_seed: int):
+    """§8.1 step (3) (L631): the dyn_index-th eligible, not-predicated-out dynamic instruction of
+    `thread` in a warp-major record stream -> dict(record, site, target ('gpr' | 'mem' | 'pred' |
+    'cc'), before, bit), or None when the thread has fewer. See oracle.cpp (reading R23)."""
+    sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+    hdr = np.ascontiguousarray(hdr, dtype=HDR_DTYPE)
+    val = None if val is None else np.ascontiguousarray(val, np.uint32)
+    out = np.zeros(5, np.uint64)
+    rc = lib().oracle_locate_injection(sites.ctypes.data, len(sites), _ptr(hdr), len(hdr), _ptr(val),
+                                       thread, dyn_index, reg_seed & 0xFFFFFFFF,
+                                       bit_seed & 0xFFFFFFFF, out.ctypes.data)
+    if rc != 0:
+        return None
+    return {"record": int(out[0]), "site": int(out[1]),
+            "target": ("gpr", "mem", "pred", "cc")[int(out[2])], "before": int(out[3]),
+            "bit": int(out[4])}

@@ -67,6 +67,7 @@ SIGNATURES = {
     "sassi_ik_trace_totals": (_i, [_vp, ctypes.POINTER(_u64), ctypes.POINTER(_u64), ctypes.POINTER(_u64)]),
     "sassi_ik_trace_copy": (_i, [_vp, _vp, _vp, _vp, _vp]),
     "sassi_ik_output_checksum": (_i, [_vp, ctypes.POINTER(_u64)]),
+    "sassi_ik_inject": (_i, [_vp, _vp, _u32, _vp, _vp]),
     "sassi_strerror": (ctypes.c_char_p, [_i]),
     "sassi_last_error": (ctypes.c_char_p, []),
 }
@@ -324,6 +325,22 @@ def sassi_ik_output_checksum(ik: int) -> int:
     return c.value
 
 
+# error-injection outcomes (include/sassi_ik.h)
+SASSI_INJ_MASKED, SASSI_INJ_SDC, SASSI_INJ_DUE, SASSI_INJ_HANG, SASSI_INJ_NOT_REACHED = range(5)
+INJ_OUTCOME_NAMES = ("masked", "sdc", "due", "hang", "not_reached")
+OUTCOME_DTYPE = np.dtype([("outcome", "<u4"), ("site", "<u4"), ("target", "<u4"), ("bit", "<u4"),
+                          ("before", "<u4"), ("after", "<u4"), ("reserved", "<u4", (2,))])
+assert OUTCOME_DTYPE.itemsize == 32
+
+
+def sassi_ik_inject(ik: int, sites: np.ndarray, stream=None) -> np.ndarray:
+    sites = np.ascontiguousarray(sites, dtype=INJ_DTYPE)
+    out = np.zeros(len(sites), dtype=OUTCOME_DTYPE)
+    _check(lib().sassi_ik_inject(ik, sites.ctypes.data if len(sites) else None, len(sites),
+                                 out.ctypes.data if len(sites) else None, _stream(stream)))
+    return out
+
+
 class InstrumentedKernel:
     """A synthetic kernel with hand-placed SASSI sites (vecadd / bfs / sgemm / stencil)."""
 
@@ -341,6 +358,21 @@ class InstrumentedKernel:
 
     def run(self, mode: int, ctx: Context | None = None, stream=None) -> None:
         sassi_ik_run(self.handle, mode, ctx.handle if ctx is not None else None, stream)
+
+    def inject(self, sites: np.ndarray, stream=None) -> np.ndarray:
+        """One error-injection run per site tuple (§8.1) -> OUTCOME_DTYPE records."""
+        return sassi_ik_inject(self.handle, sites, stream)
+
+    def injection_campaign(self, k: int = 1000, seed: int = 20150616, stream=None):
+        """§8.1's three steps on this kernel: (1) profile the per-thread eligible counts,
+        (2) draw k injection sites, (3) one injection run per site. -> (sites, outcomes)."""
+        ctx = self.context(SASSI_H_INSTCOUNT)
+        try:
+            self.run(SASSI_H_INSTCOUNT, ctx, stream)
+            sites = ctx.sample(k, seed, stream)
+        finally:
+            ctx.close()
+        return sites, self.inject(sites, stream)
 
     def checksum(self) -> int:
         return sassi_ik_output_checksum(self.handle)
