@@ -308,3 +308,32 @@ def test_c5_full_shard_sampled_warps_exact():
     ctx.consume(dict(d, hdr=d["hdr"][half:], chunk_base=d["chunk_base"][half // 256:], n=d["n"] - half))
     assert np.array_equal(ctx.read_tables(), full)
     ctx.close()
+
+
+def test_permuted_records_give_identical_tables():
+    """§4.2 item 5: every table is a commutative fold — shuffling whole records (with their rows)
+    across chunks and batches changes nothing, on the GPU as in the oracle."""
+    from test_oracle import permute_records
+    s, W, hdr, addr, val = random_trace(2024, n=6000)
+    o = oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val)
+    for seed in (1, 2):
+        h2, a2, v2 = permute_records(s, hdr, addr, val, seed)
+        t = gpu_table(s, W, sassi.SASSI_H_EVERY, to_device(s, h2, a2, v2))
+        assert diff_tables(t, o, len(s), W) is None
+
+
+def test_virtual_ranks_merged_on_host_equal_single_pass():
+    """§4.2 item 8 (multi-GPU without a cluster): P shards consumed into P contexts on one GPU,
+    merged with the oracle's merge, equal the unsharded fold."""
+    from test_oracle import _split
+    s, W, hdr, addr, val = random_trace(99, n=9000)
+    single = gpu_table(s, W, sassi.SASSI_H_EVERY, to_device(s, hdr, addr, val))
+    acc = oracle.table_init(len(s), W, sassi.SASSI_H_EVERY)
+    parts = []
+    for half in _split(s, hdr, addr, val, 4000):
+        parts += _split(s, *half, len(half[0]) // 3)
+    for h, a, v in parts:
+        t = gpu_table(s, W, sassi.SASSI_H_EVERY, to_device(s, h, a, v))
+        oracle.merge(acc, t, len(s), W)
+    assert diff_tables(acc, single, len(s), W) is None
+    assert np.array_equal(single, oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val))
