@@ -1,6 +1,7 @@
 // common.cuh — internals shared by the libsassi.so translation units (never by the oracle).
 #pragma once
 
+#include <nvtx3/nvToolsExt.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -10,6 +11,14 @@
 #include "sassi.h"
 
 namespace sassi {
+
+// NVTX range around a public call (header-only nvtx3: no cost unless a profiler is attached)
+struct NvtxRange {
+  explicit NvtxRange(const char* m) { nvtxRangePushA(m); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr uint32_t EMPTY_KEY = 0xFFFFFFFFu;
