@@ -67,6 +67,10 @@
  *   mix[S]         thread executions per site: sum of popc(active) (Fig.3's count, per site)
  *   imix[8]        Fig.3's dynamic_instr_counts[7] = {memory, extended memory (width > 4 B),
  *                  controlxfer, sync, numeric, texture, total executed}, then one zero word
+ *   pcsel[4]       sites whose per-PC memdiv matrix is kept: site index + 1 (0 = slot unused);
+ *                  configuration (sassi_select_memdiv_pcs), not a counter
+ *   pcmat[4][32][32]  per selected pc, the h32 matrix of its own records (L353 "detailed
+ *                  accounting of unique references generated per program counter")
  *
  * ---------------------------------------------------------------------------------------------
  * CONVENTIONS
@@ -87,11 +91,12 @@
 extern "C" {
 #endif
 
-#define SASSI_ABI_VERSION 2u
+#define SASSI_ABI_VERSION 3u
 #define SASSI_WARP_SIZE 32u
 #define SASSI_CHUNK 256u           /* records per chunk_base entry */
 #define SASSI_MAX_SITES 4096u      /* registered sites per context */
 #define SASSI_MAX_DST 4u           /* GPR destinations per instruction (e.g. 128-bit loads) */
+#define SASSI_MAX_PC_MATRICES 4u   /* per-PC memdiv matrices (sassi_select_memdiv_pcs)          */
 
 typedef enum sassi_status {
   SASSI_OK = 0,
@@ -168,7 +173,8 @@ typedef struct sassi_inj_site {
 } sassi_inj_site;      /* 32 B */
 
 typedef struct sassi_layout {
-  uint64_t diag, br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, total; /* u64 words */
+  uint64_t diag, br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, pcsel, pcmat,
+      total; /* u64 words */
 } sassi_layout;
 
 /* Offsets of the table image (host-only arithmetic; no device needed). */
@@ -186,6 +192,14 @@ void sassi_ctx_destroy(struct sassi_ctx* ctx);
  * (L181-L187). Allowed only
  * before the first consume or right after sassi_reset. Errors: EINVAL, ESTATE, ENOSPC. */
 int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
+
+/* Keep a per-PC memory-divergence matrix (pcmat, the Fig.6 32x32 matrix of that pc's own records)
+ * for k <= SASSI_MAX_PC_MATRICES registered GLOBAL memory sites given by pc (HOST array; k = 0
+ * clears the selection). Like sassi_attach_handler: only before the first consume or right after
+ * sassi_reset; the selection is part of the site-table checksum sassi_merge compares. Takes
+ * effect with SASSI_H_MEMDIV attached; costs 4 KB of shared memory per selected pc per CTA.
+ * Errors: EINVAL (unknown pc, not a GLOBAL memory site, k too large), ESTATE, ENOSPC. */
+int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
 
 /* Fold n records (DEVICE buffers) into the context's tables; asynchronous, stream-ordered.
  * Tables accumulate across calls until sassi_reset. Errors: EINVAL, ESTATE (no handler), ECUDA. */

@@ -54,7 +54,9 @@ def layout(n_sites: int, n_warps: int) -> dict:
     L["counts"] = L["h128"] + 1024
     L["mix"] = L["counts"] + 32 * W
     L["imix"] = L["mix"] + S
-    L["total"] = L["imix"] + 8
+    L["pcsel"] = L["imix"] + 8
+    L["pcmat"] = L["pcsel"] + 4
+    L["total"] = L["pcmat"] + 4 * 1024
     return L
 
 
@@ -75,7 +77,9 @@ def sections(table: np.ndarray, n_sites: int, n_warps: int) -> dict:
         "h128": t[L["h128"]:L["counts"]].reshape(32, 32),
         "counts": t[L["counts"]:L["mix"]],
         "mix": t[L["mix"]:L["imix"]],
-        "imix": t[L["imix"]:L["total"]],
+        "imix": t[L["imix"]:L["pcsel"]],
+        "pcsel": t[L["pcsel"]:L["pcmat"]],
+        "pcmat": t[L["pcmat"]:L["total"]].reshape(4, 32, 32),
     }
 
 
@@ -110,6 +114,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_sample.restype = ctypes.c_int
         L.oracle_splitmix64.argtypes = [u64]
         L.oracle_splitmix64.restype = u64
+        L.oracle_select_pcs.argtypes = [u32, u32, vp, u32, vp]
+        L.oracle_select_pcs.restype = None
         L.oracle_locate_injection.argtypes = [vp, u32, vp, u64, vp, u64, u64, u32, u32, vp]
         L.oracle_locate_injection.restype = ctypes.c_int
         _lib = L
@@ -120,10 +126,14 @@ def _ptr(a):
     return None if a is None or a.size == 0 else a.ctypes.data
 
 
-def table_init(n_sites: int, n_warps: int, handler_mask: int) -> np.ndarray:
+def table_init(n_sites: int, n_warps: int, handler_mask: int, pcs=()) -> np.ndarray:
+    """Fresh table; `pcs` = up to 4 site indices whose per-PC memdiv matrices are kept."""
     L = lib()
     t = np.zeros(int(L.oracle_table_words(n_sites, n_warps)), dtype=np.uint64)
     L.oracle_table_init(n_sites, n_warps, handler_mask, t.ctypes.data)
+    if len(pcs):
+        sel = np.ascontiguousarray(pcs, dtype=np.uint32)
+        L.oracle_select_pcs(n_sites, n_warps, sel.ctypes.data, len(sel), t.ctypes.data)
     return t
 
 
@@ -147,9 +157,9 @@ def consume(table: np.ndarray, sites: np.ndarray, n_warps: int, handler_mask: in
     return table
 
 
-def run(sites, n_warps, handler_mask, hdr, addr=None, val=None) -> np.ndarray:
+def run(sites, n_warps, handler_mask, hdr, addr=None, val=None, pcs=()) -> np.ndarray:
     """Fresh table + one consume."""
-    t = table_init(len(sites), n_warps, handler_mask)
+    t = table_init(len(sites), n_warps, handler_mask, pcs)
     return consume(t, sites, n_warps, handler_mask, hdr, addr, val)
 
 

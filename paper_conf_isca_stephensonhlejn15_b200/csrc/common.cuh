@@ -34,6 +34,8 @@ constexpr uint32_t I_MEMDIV = 1u << 2;        // MEM && GLOBAL: folded by the me
 constexpr uint32_t I_ELIGIBLE = 1u << 3;      // instcount-eligible (R12)
 constexpr uint32_t I_NDST_SHIFT = 4;          // 3 bits: n_gpr_dst
 constexpr uint32_t I_VD0_SHIFT = 8;           // 16 bits: first value-destination state slot
+constexpr uint32_t I_PCM = 1u << 24;          // memdiv site with a per-PC matrix ...
+constexpr uint32_t I_PCM_SHIFT = 25;          // ... in slot (info >> 25) & 3
 
 // Home slot of a pc in the site hash: multiplicative hash ((pc * mul) >> shr) & (cap - 1), its
 // parameters chosen per site table at attach time (capi.cu choose_hash): for the dense pcs of a
@@ -45,7 +47,7 @@ __host__ __device__ __forceinline__ uint32_t pc_slot(uint32_t pc, uint32_t mul, 
 
 // Table image offsets (u64 words), same formulas as sassi_table_layout().
 struct Offsets {
-  uint64_t br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, total;
+  uint64_t br, mem, val, ones, zeros, scalar, h32, h128, counts, mix, imix, pcsel, pcmat, total;
 };
 
 // Kernel parameter block of the fused consume kernel.
@@ -70,6 +72,7 @@ struct ConsumeParams {
   const uint32_t* flush_x;          // [S] Fig.3 category bits of each site (instruction mix)
   uint32_t S;                       // registered sites
   uint32_t px;                      // first private word of the per-site mix counters
+  uint32_t npcm;                    // per-PC memdiv matrices kept (shared-memory copies)
   uint64_t* table;                  // device table image
   Offsets off;
   uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
@@ -96,6 +99,9 @@ struct sassi_ctx {
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t pw_base = 0;             // private words of the branch / memdiv / value counters
   std::vector<uint32_t> mix_cat;    // per site: Fig.3 category bits (bit c = dynamic_instr_counts[c])
+  uint32_t pcsel[4] = {0, 0, 0, 0}; // per-PC memdiv matrices: site index + 1 (0 = unused)
+  uint32_t npcm = 0;
+  uint64_t site_checksum = 0;       // of the registered sites (checksum adds the selection)
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
   uint32_t* d_err = nullptr;
   uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums

@@ -202,6 +202,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
   uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
   uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + (Ly::kVal ? p.nvd : 0u));  // counters
+  uint32_t* s_pcm = s_priv + (p.priv ? kWarpsPerCta : 1u) * p.pw;  // [npcm][32][32] per-PC matrices
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
 
   const uint32_t tid = threadIdx.x;
@@ -211,6 +212,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
   if (H & kCounters)
     for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
   for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
+  if (H & SASSI_H_MEMDIV)
+    for (uint32_t i = tid; i < 1024 * p.npcm; i += blockDim.x) s_pcm[i] = 0;
   if (Ly::kVal && tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
@@ -416,6 +419,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
           if (selm_l) {
             atomicAdd(sm + kSmH32 + 32 * (n - 1) + (my_s - 1), 1u);
             atomicAdd(sm + kSmH128 + 32 * (n - 1) + (my_l - 1), 1u);
+            if (info & I_PCM)  // this pc's own matrix (sassi_select_memdiv_pcs)
+              atomicAdd(s_pcm + 1024 * ((info >> I_PCM_SHIFT) & 3u) + 32 * (n - 1) + (my_s - 1), 1u);
           }
           add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv);
         }
@@ -426,7 +431,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
         add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv);
         if (vtot) {
           const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
-          const uint32_t vslot = info >> I_VD0_SHIFT;         // its first value-state slot
+          const uint32_t vslot = (info >> I_VD0_SHIFT) & 0xFFFFu;  // its first value-state slot
           for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
             const uint32_t nr = min(vtot - s0, 32u);
             if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
@@ -543,6 +548,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       const uint32_t v = sm[kSmH32 + c];
       if (v) atomicAdd(table + (c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024)), (unsigned long long)v);
     }
+    for (uint32_t c = tid; c < 1024 * p.npcm; c += blockDim.x)
+      if (s_pcm[c]) atomicAdd(table + p.off.pcmat + c, (unsigned long long)s_pcm[c]);
   }
   if (H & SASSI_H_INSTMIX) {
     unsigned long long* const s_imix = reinterpret_cast<unsigned long long*>(sm + kSmImix);
@@ -607,6 +614,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   if (H & SASSI_H_VALUE) words += 4ull * c->nvd;
   if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX))
     words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
+  if (H & SASSI_H_MEMDIV) words += 1024ull * c->npcm;  // per-PC matrices
   *bytes = 4 * words;
   return 0;
 }

@@ -70,16 +70,17 @@ int nccl_err(ncclResult_t r, const char* what) {
   return set_error(SASSI_ENCCL, std::string(what) + ": " + nccl().GetErrorString(r));
 }
 
-// packed image: [4 diag][br..val sums][h32..counts sums][isScalar 0/1 sums, 4S][ones+zeros masks
-// byte-expanded, 8S x 4 words]. After the sum: isScalar = (sum == nranks); mask bit set iff its
-// byte == nranks.
+// packed image: [4 diag][br..val sums][h32..imix sums, then pcmat sums][isScalar 0/1 sums, 4S]
+// [ones+zeros masks byte-expanded, 8S x 4 words]. After the sum: isScalar = (sum == nranks); mask
+// bit set iff its byte == nranks. pcsel (configuration, equal on every rank) is not packed.
 struct PackLayout {
-  uint64_t n_sum_a, n_sum_b, n_scalar, n_mask_words, total;
+  uint64_t n_sum_a, n_sum_b1, n_sum_b, n_scalar, n_mask_words, total;
 };
 PackLayout pack_layout(const sassi_ctx* c) {
   PackLayout L;
   L.n_sum_a = c->off.ones - c->off.br;
-  L.n_sum_b = c->off.total - c->off.h32;
+  L.n_sum_b1 = c->off.pcsel - c->off.h32;
+  L.n_sum_b = L.n_sum_b1 + (c->off.total - c->off.pcmat);
   L.n_scalar = 4ull * c->S;
   L.n_mask_words = 8ull * c->S * 4;
   L.total = 4 + L.n_sum_a + L.n_sum_b + L.n_scalar + L.n_mask_words;
@@ -93,7 +94,8 @@ __global__ void pack_kernel(const uint64_t* __restrict__ t, Offsets o, PackLayou
     uint64_t v;
     if (i < 4) v = t[i];
     else if (i < b1) v = t[o.br + (i - 4)];
-    else if (i < b2) v = t[o.h32 + (i - b1)];
+    else if (i < b1 + L.n_sum_b1) v = t[o.h32 + (i - b1)];
+    else if (i < b2) v = t[o.pcmat + (i - b1 - L.n_sum_b1)];
     else if (i < b3) v = t[o.scalar + (i - b2)];
     else {
       const uint64_t w = i - b3;
@@ -115,7 +117,8 @@ __global__ void unpack_kernel(uint64_t* __restrict__ t, Offsets o, PackLayout L,
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_items; i += stride) {
     if (i < 4) t[i] = pk[i];
     else if (i < b1) t[o.br + (i - 4)] = pk[i];
-    else if (i < b2) t[o.h32 + (i - b1)] = pk[i];
+    else if (i < b1 + L.n_sum_b1) t[o.h32 + (i - b1)] = pk[i];
+    else if (i < b2) t[o.pcmat + (i - b1 - L.n_sum_b1)] = pk[i];
     else if (i < b3) t[o.scalar + (i - b2)] = pk[i] == nranks ? 1ull : 0ull;
     else {
       const uint64_t m = i - b3;

@@ -16,7 +16,9 @@ Offsets layout_offsets(uint32_t S, uint32_t W) {
   o.counts = o.h128 + 1024;
   o.mix = o.counts + 32ull * W;
   o.imix = o.mix + S;
-  o.total = o.imix + 8;
+  o.pcsel = o.imix + 8;
+  o.pcmat = o.pcsel + 4;
+  o.total = o.pcmat + 4ull * 1024;
   return o;
 }
 
@@ -25,7 +27,8 @@ namespace {
 // Sums start at 0; constantOnes / constantZeros start all-ones and isScalar starts 1 (the AND
 // identities, Fig.9);
 // diag[4..7] describe the image.
-__global__ void init_tables_kernel(uint64_t* t, Offsets o, uint32_t S, uint32_t W, uint32_t mask) {
+__global__ void init_tables_kernel(uint64_t* t, Offsets o, uint32_t S, uint32_t W, uint32_t mask,
+                                   uint4 pcsel) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < o.total; i += stride) {
     uint64_t v = 0;
@@ -35,6 +38,10 @@ __global__ void init_tables_kernel(uint64_t* t, Offsets o, uint32_t S, uint32_t 
     else if (i == 5) v = W;
     else if (i == 6) v = mask;
     else if (i == 7) v = SASSI_ABI_VERSION;
+    else if (i == o.pcsel) v = pcsel.x;
+    else if (i == o.pcsel + 1) v = pcsel.y;
+    else if (i == o.pcsel + 2) v = pcsel.z;
+    else if (i == o.pcsel + 3) v = pcsel.w;
     t[i] = v;
   }
 }
@@ -44,7 +51,8 @@ __global__ void init_tables_kernel(uint64_t* t, Offsets o, uint32_t S, uint32_t 
 int launch_init_tables(sassi_ctx* c, cudaStream_t s) {
   uint64_t blocks = (c->off.total + 255) / 256;
   if (blocks > 4096) blocks = 4096;
-  init_tables_kernel<<<(unsigned)blocks, 256, 0, s>>>(c->d_table, c->off, c->S, c->W, c->mask);
+  const uint4 sel = make_uint4(c->pcsel[0], c->pcsel[1], c->pcsel[2], c->pcsel[3]);
+  init_tables_kernel<<<(unsigned)blocks, 256, 0, s>>>(c->d_table, c->off, c->S, c->W, c->mask, sel);
   SASSI_CUDA(cudaGetLastError());
   c->launches += 1;
   return SASSI_OK;
@@ -67,6 +75,8 @@ extern "C" int sassi_table_layout(uint32_t n_sites, uint32_t n_warps, sassi_layo
   out->counts = o.counts;
   out->mix = o.mix;
   out->imix = o.imix;
+  out->pcsel = o.pcsel;
+  out->pcmat = o.pcmat;
   out->total = o.total;
   return SASSI_OK;
 }

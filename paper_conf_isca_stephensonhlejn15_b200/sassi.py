@@ -40,7 +40,7 @@ class SassiRecords(ctypes.Structure):
 
 class SassiLayout(ctypes.Structure):
     _fields_ = [(k, _u64) for k in ("diag", "br", "mem", "val", "ones", "zeros", "scalar", "h32",
-                                    "h128", "counts", "mix", "imix", "total")]
+                                    "h128", "counts", "mix", "imix", "pcsel", "pcmat", "total")]
 
 
 SIGNATURES = {
@@ -48,6 +48,7 @@ SIGNATURES = {
     "sassi_ctx_create": (_i, [ctypes.POINTER(_vp), _i, _vp, _u32, _u32]),
     "sassi_ctx_destroy": (None, [_vp]),
     "sassi_attach_handler": (_i, [_vp, _u32]),
+    "sassi_select_memdiv_pcs": (_i, [_vp, _vp, _u32]),
     "sassi_consume": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_consume_host": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_index_records": (_i, [_vp, _vp, _u64, _vp, _vp]),
@@ -161,6 +162,11 @@ def sassi_attach_handler(ctx: int, kind_mask: int) -> None:
     _check(lib().sassi_attach_handler(ctx, kind_mask))
 
 
+def sassi_select_memdiv_pcs(ctx: int, pcs) -> None:
+    a = np.ascontiguousarray(pcs, dtype=np.uint32)
+    _check(lib().sassi_select_memdiv_pcs(ctx, a.ctypes.data if a.size else None, a.size))
+
+
 def sassi_consume(ctx: int, rec: dict, n=None, stream=None) -> None:
     n = rec["n"] if n is None else n
     r = _records(rec)
@@ -250,6 +256,10 @@ class Context:
     def reset(self, stream=None):
         sassi_reset(self.handle, stream)
 
+    def select_memdiv_pcs(self, pcs) -> None:
+        """Keep per-PC memory-divergence matrices (pcmat) for up to 4 GLOBAL memory sites."""
+        sassi_select_memdiv_pcs(self.handle, pcs)
+
     def read_tables(self, stream=None) -> np.ndarray:
         return sassi_read_tables(self.handle, self.layout["total"], stream)
 
@@ -263,7 +273,9 @@ class Context:
                 "scalar": t[L["scalar"]:L["h32"]].reshape(S, 4),
                 "h32": t[L["h32"]:L["h128"]].reshape(32, 32),
                 "h128": t[L["h128"]:L["counts"]].reshape(32, 32), "counts": t[L["counts"]:L["mix"]],
-                "mix": t[L["mix"]:L["imix"]], "imix": t[L["imix"]:L["total"]]}
+                "mix": t[L["mix"]:L["imix"]], "imix": t[L["imix"]:L["pcsel"]],
+                "pcsel": t[L["pcsel"]:L["pcmat"]],
+                "pcmat": t[L["pcmat"]:L["total"]].reshape(4, 32, 32)}
 
     def sample(self, k: int, seed: int, stream=None) -> np.ndarray:
         return sassi_sample_sites(self.handle, k, seed, stream)

@@ -39,9 +39,12 @@ def to_device(sites, hdr, addr, val, chunk_base=None):
                 n=len(hdr), n_addr_rows=len(addr), n_val_rows=len(val))
 
 
-def gpu_table(sites, n_warps, mask, drec, n=None):
+def gpu_table(sites, n_warps, mask, drec, n=None, pcs=()):
+    """One consume through the C ABI; `pcs` = pcs of the per-PC memdiv matrices to keep."""
     ctx = sassi.Context(sites, n_warps, mask)
     try:
+        if len(pcs):
+            ctx.select_memdiv_pcs(pcs)
         ctx.consume(drec, n)
         return ctx.read_tables()
     finally:

@@ -21,18 +21,21 @@ def pack(t, S, W):
     masks = t[L["ones"]:L["scalar"]].astype(np.uint32)               # ones[S][4], zeros[S][4]
     bits = np.unpackbits(masks.view(np.uint8).reshape(-1, 4), axis=1, bitorder="little")
     expanded = bits.astype(np.uint8).reshape(-1, 32).view(np.uint64).reshape(-1)  # 4 words / mask
-    return np.concatenate([t[0:4], t[L["br"]:L["ones"]], t[L["h32"]:L["total"]],
-                           t[L["scalar"]:L["h32"]], expanded]).astype(np.uint64)
+    return np.concatenate([t[0:4], t[L["br"]:L["ones"]], t[L["h32"]:L["pcsel"]],
+                           t[L["pcmat"]:L["total"]], t[L["scalar"]:L["h32"]],
+                           expanded]).astype(np.uint64)
 
 
 def unpack(pk, t, S, W, nranks):
     L = oracle.layout(S, W)
     out = t.copy()
     a = L["ones"] - L["br"]
-    b = L["total"] - L["h32"]
+    b1 = L["pcsel"] - L["h32"]
+    b = b1 + (L["total"] - L["pcmat"])               # the pc selection (pcsel) is not summed
     out[0:4] = pk[0:4]
     out[L["br"]:L["ones"]] = pk[4:4 + a]
-    out[L["h32"]:L["total"]] = pk[4 + a:4 + a + b]
+    out[L["h32"]:L["pcsel"]] = pk[4 + a:4 + a + b1]
+    out[L["pcmat"]:L["total"]] = pk[4 + a + b1:4 + a + b]
     out[L["scalar"]:L["h32"]] = (pk[4 + a + b:4 + a + b + 4 * S] == nranks).astype(np.uint64)
     bytes_ = pk[4 + a + b + 4 * S:].view(np.uint8).reshape(-1, 32)
     bits = (bytes_ == nranks).astype(np.uint8)

@@ -261,7 +261,10 @@ def test_merge_single_rank_nccl():
     leave the tables unchanged (sums over one rank; masks survive the byte-expansion round trip)."""
     s, W, hdr, addr, val = random_trace(555, n=6000)
     d = to_device(s, hdr, addr, val)
-    ctx = sassi.Context(s, W, sassi.SASSI_H_ALL)
+    ctx = sassi.Context(s, W, sassi.SASSI_H_EVERY)
+    sel = [i for i in range(len(s)) if (int(s[i]["flags"]) & oracle.F_MEM)
+           and int(s[i]["domain"]) == oracle.D_GLOBAL][:4]
+    ctx.select_memdiv_pcs([int(s[i]["pc"]) for i in sel])
     ctx.consume(d)
     before = ctx.read_tables()
     uid = sassi.sassi_nccl_get_unique_id()
@@ -271,7 +274,7 @@ def test_merge_single_rank_nccl():
     sassi.sassi_nccl_comm_destroy(comm)
     ctx.close()
     assert np.array_equal(after, before)
-    assert np.array_equal(after, oracle.run(s, W, oracle.H_ALL, hdr, addr, val))
+    assert np.array_equal(after, oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val, pcs=sel))
 
 
 def test_c5_full_shard_sampled_warps_exact():
@@ -337,3 +340,59 @@ def test_virtual_ranks_merged_on_host_equal_single_pass():
         oracle.merge(acc, t, len(s), W)
     assert diff_tables(acc, single, len(s), W) is None
     assert np.array_equal(single, oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val))
+
+
+def _global_mem_sites(s):
+    return [i for i in range(len(s)) if (int(s[i]["flags"]) & oracle.F_MEM)
+            and int(s[i]["domain"]) == oracle.D_GLOBAL]
+
+
+@pytest.mark.parametrize("mask", [2, 15, 31])
+def test_per_pc_memdiv_matrices_t0(mask):
+    s = T0.sites()
+    hdr, addr, val = T0.records()
+    t = gpu_table(s, T0.N_WARPS, mask, to_device(s, hdr, addr, val), pcs=[0x30, 0x20])
+    o = oracle.run(s, T0.N_WARPS, mask, hdr, addr, val, pcs=[2, 1])
+    assert diff_tables(t, o, len(s), T0.N_WARPS) is None
+    sec = oracle.sections(t, len(s), T0.N_WARPS)
+    assert list(map(int, sec["pcsel"])) == [3, 2, 0, 0]
+    assert np.array_equal(sec["pcmat"][0] + sec["pcmat"][1], sec["h32"])
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_per_pc_memdiv_matrices_random(seed):
+    s, W, hdr, addr, val = random_trace(3000 + seed, n=8000)
+    sel = _global_mem_sites(s)[:4]
+    o = oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val, pcs=sel)
+    t = gpu_table(s, W, sassi.SASSI_H_EVERY, to_device(s, hdr, addr, val),
+                  pcs=[int(s[i]["pc"]) for i in sel])
+    assert diff_tables(t, o, len(s), W) is None
+
+
+def test_per_pc_memdiv_matrices_c2_full():
+    """c2 (10^7 records) with four selected gather / unit-stride sites."""
+    P, mask, d = _gen("c2")
+    h = gen.to_host(d)
+    sel = _global_mem_sites(h["sites"])[:4]
+    t = gpu_table(h["sites"], P.total_warps, mask, d, pcs=[int(h["sites"][i]["pc"]) for i in sel])
+    o = oracle.run(h["sites"], P.total_warps, mask, h["hdr"], h["addr"], h["val"], pcs=sel)
+    assert diff_tables(t, o, len(h["sites"]), P.total_warps) is None
+    assert oracle.sections(t, len(h["sites"]), P.total_warps)["pcmat"].sum() > 0
+
+
+def test_select_memdiv_pcs_errors():
+    s = T0.sites()
+    ctx = sassi.Context(s, T0.N_WARPS, 2)
+    for bad in ([0x40], [0x50], [0x999], [0x20, 0x20], [0x20, 0x30, 0x20, 0x30, 0x20]):
+        with pytest.raises(sassi.SassiError) as e:   # ALU, shared-memory, unregistered, twice, > 4
+            ctx.select_memdiv_pcs(bad)
+        assert e.value.status == sassi.SASSI_EINVAL
+    hdr, addr, val = T0.records()
+    ctx.consume(to_device(s, hdr, addr, val))
+    with pytest.raises(sassi.SassiError) as e:
+        ctx.select_memdiv_pcs([0x20])
+    assert e.value.status == sassi.SASSI_ESTATE
+    ctx.reset()
+    ctx.select_memdiv_pcs([0x20])
+    ctx.select_memdiv_pcs([])
+    ctx.close()

@@ -25,6 +25,8 @@ for mask in (1, 2, 4, 8, 15, 16, 31):
 s2, W, h2, a2, v2 = random_trace(4321, n=3000)
 t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2))
 assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2))
+t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2), pcs=[int(s2[1]["pc"]), int(s2[7]["pc"])])
+assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2, pcs=[1, 7]))
 P, lim, mask, _ = gen.preset("c1")
 dc = gen.generate_device(P, lim)
 ctx = sassi.Context(dc["sites"], P.total_warps, 31)
