@@ -36,14 +36,25 @@ __device__ __forceinline__ uint64_t ld_nc_u64(const uint64_t* p) {
   return r;
 }
 // 32x32 bit-matrix transpose across the warp: in, lane i holds row i; out, lane l holds the word
-// whose bit i is bit l of row i. Five butterfly stages swapping off-diagonal blocks.
+// whose bit i is bit l of row i. Five butterfly stages swapping off-diagonal blocks: per stage the
+// lane keeps its own half (mask `keep`) and takes the partner's other half, brought into place by
+// one rotate (right by J in the upper lane of a pair, left by J in the lower: the wrapped bits fall
+// outside the taken half). The rotate form issues fewer instructions but holds more registers: the
+// header-only kernels use it, the payload kernels (register-capped at 64) the shift form.
+template <bool kRotate>
 __device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
   const uint32_t m16 = 0x0000FFFFu, m8 = 0x00FF00FFu, m4 = 0x0F0F0F0Fu, m2 = 0x33333333u,
                  m1 = 0x55555555u;
-#define SASSI_TSTAGE(J, M)                                              \
-  {                                                                     \
-    uint32_t y = __shfl_xor_sync(FULL, x, J);                           \
-    x = (lane & J) ? ((x & ~M) | ((y >> J) & M)) : ((x & M) | ((y << J) & ~M)); \
+#define SASSI_TSTAGE(J, M)                                                           \
+  {                                                                                  \
+    const uint32_t y = __shfl_xor_sync(FULL, x, J);                                  \
+    const bool hi = (lane & J) != 0;                                                 \
+    if (kRotate) {                                                                   \
+      const uint32_t keep = hi ? ~M : M;                                             \
+      x = (x & keep) | (__funnelshift_r(y, y, hi ? J : 32u - J) & ~keep);            \
+    } else {                                                                         \
+      x = hi ? ((x & ~M) | ((y >> J) & M)) : ((x & M) | ((y << J) & ~M));            \
+    }                                                                                \
   }
   SASSI_TSTAGE(16, m16)
   SASSI_TSTAGE(8, m8)
@@ -231,24 +242,135 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
   uint32_t acc = 0, acc_w = FULL;  // per-thread-count accumulator of trace warp acc_w, lane = lane
   // vertical (bit-sliced) counters: lane r's bit l of plane k is bit k of the number of batches in
   // which lane r's record had lane l eligible (records of trace warp acc_w only); transposed and
-  // folded into acc every 7 batches, so most batches cost 5 LOPs instead of a 32x32 transpose.
+  // folded into acc every 15 batches, so most batches cost 7 LOPs instead of a 32x32 transpose.
   // Only for handler sets without payload rows: with them, the 4 extra registers cost more than
   // the transposes they save (measured: c3 2.90 -> 3.06 ms)
   constexpr bool kVertical = !(H & (SASSI_H_MEMDIV | SASSI_H_VALUE));
-  uint32_t vp0 = 0, vp1 = 0, vp2 = 0, vn = 0;
+  uint32_t vp0 = 0, vp1 = 0, vp2 = 0, vp3 = 0, vn = 0;
   auto flush_planes = [&]() {
     if (vn) {
-      acc += __popc(transpose32(vp0, lane)) + 2 * __popc(transpose32(vp1, lane)) +
-             4 * __popc(transpose32(vp2, lane));
-      vp0 = vp1 = vp2 = 0;
+      acc += __popc(transpose32<true>(vp0, lane)) + 2 * __popc(transpose32<true>(vp1, lane)) +
+             4 * __popc(transpose32<true>(vp2, lane)) + 8 * __popc(transpose32<true>(vp3, lane));
+      vp0 = vp1 = vp2 = vp3 = 0;
       vn = 0;
     }
   };
   uint32_t err = 0;
   unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
 
-  for (uint32_t u = blockIdx.x * kWarpsPerCta + wib; u < n_units; u += nw) {
-    constexpr bool kUnitRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
+  // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239). Returns the
+  // slot {key, info, cidx, site}; `known` = a registered site (0xFFFFFFFF is never registered) ----
+  // h is always a real header of the stream (loads are clamped), so the probe needs no guard;
+  // records are counted per chunk / range (c_rec), not here
+  auto lookup = [&](const uint4& h, bool valid, bool& known) -> uint4 {
+    uint32_t slot = pc_slot(h.x, p.hmul, p.hshr, cap);
+    uint4 e = s_hash[slot];
+    while (e.x != h.x && e.x != EMPTY_KEY) {  // collision: linear probing (load <= 1/2, rare)
+      slot = (slot + 1) & (cap - 1);
+      e = s_hash[slot];
+    }
+    known = valid && e.x == h.x && h.x != EMPTY_KEY;
+    c_unk += valid && !known;
+    c_inv += known && h.z == 0;
+    return e;
+  };
+  // ---- the handlers that read only the header: branch (Fig.4), instruction mix (Fig.3),
+  // per-thread counts (§8.1) ----
+  auto header_handlers = [&](const uint4& h, uint32_t info, uint32_t cidx, uint32_t site, bool live,
+                             uint32_t G) {
+    const uint32_t act = h.z;
+    // ---- Case study I: branch divergence (Fig.4) ----
+    if (H & SASSI_H_BRANCH) {
+      const bool isb = live && (info & I_BRANCH);
+      add_counters4(isb, 4 * (cidx & 0xFFFFu),
+                    make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
+                               (G != 0 && G != act) ? 1u : 0u),
+                    wpriv);
+    }
+    // ---- Fig.3 instruction mix (L193-L199): every active thread counts; per-site thread
+    // executions here, the seven category totals at the flush (R22) ----
+    if ((H & SASSI_H_INSTMIX) && live) atomicAdd(wpriv + p.px + site, (uint32_t)__popc(act));
+    // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
+    if (H & SASSI_H_INSTCOUNT) {
+      uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
+      if (E != 0 && h.y >= p.n_warps) {
+        ++c_bad;
+        E = 0;
+      }
+      uint32_t pend;
+      if (kVertical) {
+        // the usual case in a warp-major stream: every eligible lane is on the accumulator's trace
+        // warp -> add E into the vertical counters (one vote decides it)
+        if (!__any_sync(FULL, E != 0 && h.y != acc_w)) {
+          const uint32_t k0 = vp0 & E;
+          vp0 ^= E;
+          const uint32_t k1 = vp1 & k0;
+          vp1 ^= k0;
+          const uint32_t k2 = vp2 & k1;
+          vp2 ^= k1;
+          vp3 ^= k2;  // at most 15 additions between flushes: no carry out of plane 3
+          if (++vn == 15) flush_planes();
+          pend = 0;
+        } else {
+          flush_planes();
+          pend = __ballot_sync(FULL, E != 0);
+        }
+      } else {
+        pend = __ballot_sync(FULL, E != 0);
+      }
+      while (pend) {
+        const uint32_t w0 = __shfl_sync(FULL, h.y, __ffs(pend) - 1);
+        const bool mine = E != 0 && h.y == w0;
+        const uint32_t cnt = __popc(transpose32<kVertical>(mine ? E : 0u, lane));
+        if (w0 != acc_w) {
+          if (acc_w != FULL && acc)
+            atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+          acc_w = w0;
+          acc = 0;
+        }
+        acc += cnt;
+        pend &= ~__ballot_sync(FULL, mine);
+        if (mine) E = 0;
+      }
+    }
+  };
+
+  constexpr bool kUnitRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
+  if (!kUnitRows) {
+    // ---- header-only handler sets: each warp takes one contiguous range of records (so its
+    // per-thread-count accumulator stays on one trace warp for thousands of records) and walks it
+    // in 32-record batches, headers loaded kDepth batches ahead ----
+    constexpr uint32_t kDepth = 3;
+    const uint32_t per = (p.n + 32u * nw - 1u) / (32u * nw) * 32u;  // records per warp
+    const uint32_t R0 = min((blockIdx.x * kWarpsPerCta + wib) * per, p.n), R1 = min(R0 + per, p.n);
+    if (lane == 0) c_rec += R1 - R0;
+    auto first_rec = [&](uint32_t t) -> uint32_t { return R0 + 32u * t; };
+    auto hload = [&](uint32_t r0) -> uint4 {
+      return r0 < R1 ? ld_nc_v4(p.hdr + min(r0 + lane, R1 - 1u)) : make_uint4(0u, 0u, 0u, 0u);
+    };
+    uint4 q[kDepth];
+#pragma unroll
+    for (uint32_t k = 0; k < kDepth; ++k) q[k] = hload(first_rec(k));
+    for (uint32_t t = 0;; t += kDepth) {
+      bool done = false;
+#pragma unroll
+      for (uint32_t k = 0; k < kDepth; ++k) {
+        const uint32_t r0 = first_rec(t + k);
+        if (r0 >= R1) {
+          done = true;
+          break;
+        }
+        const uint4 h = q[k];
+        q[k] = hload(first_rec(t + k + kDepth));
+        bool known;
+        const uint4 e = lookup(h, r0 + lane < R1, known);
+        const bool live = known && h.z != 0;
+        header_handlers(h, known ? e.y : 0u, e.z, e.w, live, h.z & h.w);
+      }
+      if (done) break;
+    }
+  }
+  for (uint32_t u = blockIdx.x * kWarpsPerCta + wib; kUnitRows && u < n_units; u += nw) {
     const ulonglong2 cb0 = kUnitRows ? p.cb[u] : make_ulonglong2(p.arow_base, p.vrow_base);
     const ulonglong2 cb1 = kUnitRows ? p.cb[u + 1] : cb0;
     if (kUnitRows && !(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end &&
@@ -264,6 +386,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
     const uint4* const hchunk = p.hdr + u * SASSI_CHUNK;
     const uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
     const uint32_t nbat = (nrec + 31) >> 5;
+    if (lane == 0) c_rec += nrec;
     // header loads are clamped to the chunk's last record (always in bounds) and masked by `valid`
     const uint32_t ilast = nrec - 1;
     uint4 hnext = ld_nc_v4(hchunk + min(lane, ilast));
@@ -273,20 +396,9 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       const bool valid = ib < nrec;
       const uint4 h = hnext;
       if (b + 1 < nbat) hnext = ld_nc_v4(hchunk + min(ib + 32, ilast));
-      // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239) ----
-      uint4 e = make_uint4(EMPTY_KEY, 0u, 0u, 0u);
-      if (valid) {
-        uint32_t slot = pc_slot(h.x, p.hmul, p.hshr, cap);
-        e = s_hash[slot];
-        while (e.x != h.x && e.x != EMPTY_KEY) {  // collision: linear probing (load <= 1/2, rare)
-          slot = (slot + 1) & (cap - 1);
-          e = s_hash[slot];
-        }
-      }
-      const bool known = valid && e.x == h.x && h.x != EMPTY_KEY;  // 0xFFFFFFFF is never registered
+      bool known;
+      const uint4 e = lookup(h, valid, known);
       const uint32_t info = known ? e.y : 0u, cidx = e.z;
-      c_rec += valid;
-      c_unk += valid && !known;
       // ---- row indices of this batch (rows follow their records); only handlers that read
       // payload rows need them, header-only handler sets skip the bookkeeping ----
       constexpr bool kRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
@@ -312,59 +424,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
       }
       const uint32_t act = h.z;
       const bool live = known && act != 0;
-      c_inv += known && act == 0;
       const uint32_t G = act & h.w;  // guard-true (or taken) active lanes
       // value rows of this batch are contiguous: start the first bulk copy now, so it lands while
       // the other handlers work on the batch
       const uint32_t* const vsrc = vchunk + 32 * vrow_b;
       if ((H & SASSI_H_VALUE) && vtot && lane == 0) bulk_load(vbuf, vsrc, 128u * min(vtot, 32u), vbar);
 
-      // ---- Case study I: branch divergence (Fig.4) ----
-      if (H & SASSI_H_BRANCH) {
-        const bool isb = live && (info & I_BRANCH);
-        add_counters4(isb, 4 * (cidx & 0xFFFFu),
-                      make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
-                                 (G != 0 && G != act) ? 1u : 0u),
-                      wpriv);
-      }
-      // ---- Fig.3 instruction mix (L193-L199): every active thread counts; per-site thread
-      // executions here, the seven category totals at the flush (R22) ----
-      if ((H & SASSI_H_INSTMIX) && live) atomicAdd(wpriv + p.px + e.w, (uint32_t)__popc(act));
-      // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
-      if (H & SASSI_H_INSTCOUNT) {
-        uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
-        if (E != 0 && h.y >= p.n_warps) {
-          ++c_bad;
-          E = 0;
-        }
-        uint32_t pend = __ballot_sync(FULL, E != 0);
-        if (kVertical && pend && __all_sync(FULL, E == 0 || h.y == acc_w)) {
-          // the usual case in a warp-major stream: add E into the vertical counters
-          const uint32_t k0 = vp0 & E;
-          vp0 ^= E;
-          const uint32_t k1 = vp1 & k0;
-          vp1 ^= k0;
-          vp2 ^= k1;  // at most 7 additions between flushes: no carry out of plane 2
-          if (++vn == 7) flush_planes();
-          pend = 0;
-        } else if (kVertical && pend) {
-          flush_planes();
-        }
-        while (pend) {
-          const uint32_t w0 = __shfl_sync(FULL, h.y, __ffs(pend) - 1);
-          const bool mine = E != 0 && h.y == w0;
-          const uint32_t cnt = __popc(transpose32(mine ? E : 0u, lane));
-          if (w0 != acc_w) {
-            if (acc_w != FULL && acc)
-              atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
-            acc_w = w0;
-            acc = 0;
-          }
-          acc += cnt;
-          pend &= ~__ballot_sync(FULL, mine);
-          if (mine) E = 0;
-        }
-      }
+      header_handlers(h, info, cidx, e.w, live, G);
       // ---- Case study II: memory address divergence (Fig.6), one warp per address row ----
       if (H & SASSI_H_MEMDIV) {
         const bool selm_l = live && (info & I_MEMDIV) && G != 0;
@@ -407,8 +473,9 @@ __global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const Consu
             const int j = __ffs(slow) - 1;
             slow &= slow - 1;
             uint32_t s, L;
-            memdiv_row64(ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j)), __shfl_sync(FULL, G, j),
-                         lane, &s, &L);
+            const uint64_t a = ld_nc_u64(abase + 32 * __shfl_sync(FULL, arel, j));
+            const uint32_t g = __shfl_sync(FULL, G, j);
+            memdiv_row64(a, g, lane, &s, &L);
             if (lane == j) {
               my_s = s;
               my_l = L;
