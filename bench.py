@@ -334,6 +334,9 @@ def main():
         comm = sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
     stream = torch.cuda.current_stream(dev)
     sample = bool(mask & 8)
+    # draws stay on the device inside the timed steps (stream-ordered, no host round trip per step)
+    draws = torch.empty(N_DRAWS * 32, dtype=torch.uint8, device=dev)
+    draw_status = torch.zeros(1, dtype=torch.int32, device=dev)
 
     def step(ev_c0=None, ev_c1=None):
         ctx.reset(stream)
@@ -345,7 +348,7 @@ def main():
         if comm is not None:
             ctx.merge(comm, stream)
         if sample:
-            ctx.sample(N_DRAWS, 20150616, stream)
+            ctx.sample_device(draws, draw_status, N_DRAWS, 20150616, stream)
 
     for _ in range(args.warmup):
         step()
@@ -367,6 +370,10 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     launches = ctx.kernel_launches() - launches0
+    if sample:   # the device-side draws of the last step == the host-output API on the same tables
+        assert int(draw_status.item()) == 0, "sampling: no eligible dynamic instruction"
+        host_draws = ctx.sample(N_DRAWS, 20150616, stream)
+        assert draws.cpu().numpy().tobytes() == host_draws.tobytes(), "device draws differ"
     ms = t_start.elapsed_time(t_end)
     consume_ms = [a.elapsed_time(b) for a, b in evs]
     if launched:

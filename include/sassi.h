@@ -228,9 +228,19 @@ int sassi_tables_device(struct sassi_ctx* ctx, const uint64_t** dev_ptr, uint64_
 
 /* Exclusive scan of the per-thread counts and k draws of injection sites (L629), uniform over
  * all eligible dynamic thread-instructions, with replacement, draw j from splitmix64(seed + j).
- * out is a HOST array of k tuples; synchronises `stream`. Errors: ESTATE if the total is 0. */
+ * out is a HOST array of k tuples; synchronises `stream` once (scan, draws and the copy back are
+ * stream-ordered with no host round trip in between). Errors: ESTATE if the total is 0 (out is
+ * then unspecified). */
 int sassi_sample_sites(struct sassi_ctx* ctx, uint32_t k, uint64_t seed, sassi_inj_site* host_out,
                        void* stream);
+
+/* The same scan and draws with DEVICE outputs and no host synchronisation (stream-ordered, so
+ * back-to-back profiling passes keep the GPU busy): dev_out[k] receives the tuples, *dev_status
+ * (device u32) is set to 0, or to 1 when the total is 0 (nothing to sample; dev_out untouched).
+ * Buffers are the caller's and must stay valid until the stream work completes.
+ * Errors: EINVAL (null pointer), ESTATE (n_warps = 0). */
+int sassi_sample_sites_device(struct sassi_ctx* ctx, uint32_t k, uint64_t seed,
+                              sassi_inj_site* dev_out, uint32_t* dev_status, void* stream);
 
 /* Multi-GPU: merge the tables of all ranks of `nccl_comm` (ncclComm_t) in place with one
  * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits).

@@ -106,6 +106,8 @@ struct sassi_ctx {
   uint32_t* d_err = nullptr;
   uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums
   uint64_t scan_words = 0;
+  void* d_sample = nullptr;         // sampling: draws + status word of the host-output form
+  uint64_t sample_bytes = 0;
   int num_sms = 0;
   int ctas_per_sm = 0;
   size_t smem_bytes = 0;
@@ -141,6 +143,8 @@ int launch_index(sassi_ctx* c, const sassi_hdr* hdr, uint64_t n, sassi_chunk_bas
                  cudaStream_t s);
 int launch_sample(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* host_out,
                   cudaStream_t s);
+int launch_sample_device(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* dev_out,
+                         uint32_t* dev_status, cudaStream_t s);
 int launch_merge(sassi_ctx* c, void* comm, cudaStream_t s);
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes);
 

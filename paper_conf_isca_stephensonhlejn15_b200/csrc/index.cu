@@ -71,7 +71,7 @@ int launch_index(sassi_ctx* c, const sassi_hdr* hdr, uint64_t n, sassi_chunk_bas
     SASSI_CUDA(cudaGetLastError());
   }
   cudaFreeAsync(buf, s);
-  c->launches += nch ? 8 : 7;
+  c->launches += nch ? 6 : 1;  // counts + 2 scans x 2 + interleave
   return rc;
 }
 

@@ -1,5 +1,5 @@
-// scan.cuh — exclusive prefix sum of a u64 array on the device (three kernels: per-block sums,
-// one-block scan of the block sums, apply). Used by sampling (per-thread counts) and by
+// scan.cuh — exclusive prefix sum of a u64 array on the device (two kernels: per-block sums, then
+// apply: each block adds up the sums of the blocks before it itself, so no third launch). Used by sampling (per-thread counts) and by
 // sassi_index_records (per-chunk row counts). Included by one .cu each (internal linkage).
 #pragma once
 #include "common.cuh"
@@ -52,27 +52,17 @@ __global__ void __launch_bounds__(kScanThreads) block_sums_kernel(const uint64_t
   if (threadIdx.x == 0) bsum[blockIdx.x] = tot;
 }
 
-__global__ void __launch_bounds__(kScanThreads) scan_bsums_kernel(uint64_t* bsum, uint64_t nb,
-                                                                  uint64_t* total_out) {
-  __shared__ uint64_t tot;
-  uint64_t carry = 0;
-  for (uint64_t b0 = 0; b0 < nb; b0 += kScanThreads) {
-    const uint64_t i = b0 + threadIdx.x;
-    const uint64_t v = i < nb ? bsum[i] : 0;
-    const uint64_t ex = block_excl_scan(v, &tot);
-    if (i < nb) bsum[i] = carry + ex;
-    carry += tot;
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) *total_out = carry;
-}
-
 __global__ void __launch_bounds__(kScanThreads) scan_apply_kernel(const uint64_t* __restrict__ c,
                                                                   uint64_t n,
                                                                   const uint64_t* __restrict__ bsum,
-                                                                  const uint64_t* total,
                                                                   uint64_t* P) {
-  __shared__ uint64_t tot;
+  __shared__ uint64_t tot, base;
+  // this block's offset: the sum of the block sums before it (a few thousand at most)
+  uint64_t part = 0;
+  for (uint64_t b = threadIdx.x; b < blockIdx.x; b += blockDim.x) part += bsum[b];
+  block_excl_scan(part, &tot);
+  if (threadIdx.x == 0) base = tot;
+  __syncthreads();
   const uint64_t i0 = blockIdx.x * kScanBlock + threadIdx.x * kScanPerThread;
   uint64_t x[kScanPerThread];
   uint64_t s = 0;
@@ -81,13 +71,13 @@ __global__ void __launch_bounds__(kScanThreads) scan_apply_kernel(const uint64_t
     x[k] = i0 + k < n ? c[i0 + k] : 0;
     s += x[k];
   }
-  uint64_t run = bsum[blockIdx.x] + block_excl_scan(s, &tot);
+  uint64_t run = base + block_excl_scan(s, &tot);
 #pragma unroll
   for (int k = 0; k < kScanPerThread; ++k) {
     if (i0 + k < n) P[i0 + k] = run;
     run += x[k];
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) P[n] = *total;
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) P[n] = base + tot;
 }
 
 }  // namespace scan_detail
@@ -95,20 +85,18 @@ __global__ void __launch_bounds__(kScanThreads) scan_apply_kernel(const uint64_t
 
 // P[0..n] = exclusive prefix of in[0..n) (P[n] = total); scratch >= scan_scratch_words(n) words.
 static inline uint64_t scan_scratch_words(uint64_t n) {
-  return (n + scan_detail::kScanBlock - 1) / scan_detail::kScanBlock + 1;
+  return (n + scan_detail::kScanBlock - 1) / scan_detail::kScanBlock;
 }
 static inline int scan_u64(const uint64_t* in, uint64_t n, uint64_t* P, uint64_t* scratch,
                            cudaStream_t s) {
   using namespace scan_detail;
   const uint64_t nb = (n + kScanBlock - 1) / kScanBlock;
-  uint64_t* total = scratch + nb;
   if (nb == 0) {
     SASSI_CUDA(cudaMemsetAsync(P, 0, 8, s));
     return SASSI_OK;
   }
   block_sums_kernel<<<(unsigned)nb, kScanThreads, 0, s>>>(in, n, scratch);
-  scan_bsums_kernel<<<1, kScanThreads, 0, s>>>(scratch, nb, total);
-  scan_apply_kernel<<<(unsigned)nb, kScanThreads, 0, s>>>(in, n, scratch, total, P);
+  scan_apply_kernel<<<(unsigned)nb, kScanThreads, 0, s>>>(in, n, scratch, P);
   SASSI_CUDA(cudaGetLastError());
   return SASSI_OK;
 }

@@ -56,6 +56,7 @@ SIGNATURES = {
     "sassi_read_tables": (_i, [_vp, _vp, _u64, _vp]),
     "sassi_tables_device": (_i, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_u64)]),
     "sassi_sample_sites": (_i, [_vp, _u32, _u64, _vp, _vp]),
+    "sassi_sample_sites_device": (_i, [_vp, _u32, _u64, _vp, _vp, _vp]),
     "sassi_merge": (_i, [_vp, _vp, _vp]),
     "sassi_nccl_get_unique_id": (_i, [_vp]),
     "sassi_nccl_comm_create": (_i, [ctypes.POINTER(_vp), _i, _i, _vp, _i]),
@@ -206,6 +207,14 @@ def sassi_sample_sites(ctx: int, k: int, seed: int, stream=None) -> np.ndarray:
     return out
 
 
+def sassi_sample_sites_device(ctx: int, k: int, seed: int, dev_out: int, dev_status: int,
+                              stream=None) -> None:
+    """Asynchronous form: k tuples to the device buffer at dev_out (32 B each), a u32 status at
+    dev_status (1 = nothing to sample)."""
+    _check(lib().sassi_sample_sites_device(ctx, k, seed & (2**64 - 1), dev_out or None, dev_status,
+                                           _stream(stream)))
+
+
 def sassi_merge(ctx: int, comm: int, stream=None) -> None:
     _check(lib().sassi_merge(ctx, comm, _stream(stream)))
 
@@ -279,6 +288,12 @@ class Context:
 
     def sample(self, k: int, seed: int, stream=None) -> np.ndarray:
         return sassi_sample_sites(self.handle, k, seed, stream)
+
+    def sample_device(self, out, status, k: int, seed: int, stream=None) -> None:
+        """Draws into `out` (a device tensor of >= 32*k bytes) and the status into `status` (a
+        device tensor of >= 4 bytes); no synchronisation."""
+        sassi_sample_sites_device(self.handle, k, seed, out.data_ptr() if k else 0,
+                                  status.data_ptr(), stream)
 
     def merge(self, comm: int, stream=None):
         sassi_merge(self.handle, comm, stream)

@@ -206,6 +206,77 @@ def test_c4_full_instcount_exact_and_sampling():
     ctx.close()
 
 
+@pytest.mark.parametrize("seed,n,n_warps", [(1, 1, 1), (2, 40, 1), (3, 700, 33), (4, 3000, 300),
+                                             (5, 20000, 1500)])
+def test_sampling_edge_cases(seed, n, n_warps):
+    """Injection-site draws (L629) against the oracle's upper_bound on the same counts: one warp
+    (33 prefix entries: the 32-ary search's last round only), prefix lengths just above a multiple
+    of 32, thousands of threads with most counts zero; k = 0 and a zero total (ESTATE)."""
+    s, W, hdr, addr, val = random_trace(3000 + seed, n=n, n_warps=n_warps)
+    mask = sassi.SASSI_H_INSTCOUNT
+    so = oracle.sections(oracle.run(s, W, mask, hdr, addr, val), len(s), W)
+    ctx = sassi.Context(s, W, mask)
+    ctx.consume(to_device(s, hdr, addr, val))
+    if int(so["counts"].sum()) == 0:
+        with pytest.raises(sassi.SassiError) as e:
+            ctx.sample(10, seed)
+        assert e.value.status == sassi.SASSI_ESTATE
+    else:
+        for k in (0, 1, 33, 1000):
+            assert np.array_equal(ctx.sample(k, seed), oracle.sample(so["counts"], k, seed))
+    ctx.reset()
+    with pytest.raises(sassi.SassiError) as e:   # nothing counted since the reset
+        ctx.sample(5, seed)
+    assert e.value.status == sassi.SASSI_ESTATE
+    ctx.close()
+
+
+def test_sampling_device_output_matches_host_output():
+    """sassi_sample_sites_device (no synchronisation, draws in device memory) == the host-output
+    form == the oracle; status 1 and outputs untouched when nothing was counted."""
+    s, W, hdr, addr, val = random_trace(5151, n=4000, n_warps=40)
+    mask = sassi.SASSI_H_INSTCOUNT
+    so = oracle.sections(oracle.run(s, W, mask, hdr, addr, val), len(s), W)
+    ctx = sassi.Context(s, W, mask)
+    ctx.consume(to_device(s, hdr, addr, val))
+    out = torch.full((300 * 32,), 0xAB, dtype=torch.uint8, device="cuda")
+    status = torch.full((1,), 7, dtype=torch.int32, device="cuda")
+    ctx.sample_device(out, status, 300, 77)
+    torch.cuda.synchronize()
+    assert int(status.item()) == 0
+    got = np.frombuffer(out.cpu().numpy().tobytes(), dtype=sassi.INJ_DTYPE)
+    assert np.array_equal(got, ctx.sample(300, 77))
+    assert np.array_equal(got, oracle.sample(so["counts"], 300, 77))
+    ctx.reset()
+    out.fill_(0xAB)
+    ctx.sample_device(out, status, 300, 77)
+    torch.cuda.synchronize()
+    assert int(status.item()) == 1 and bool((out == 0xAB).all())
+    ctx.close()
+
+
+def test_sampling_one_thread_holds_every_count():
+    """All eligible instructions on the last thread: every draw must pick it (upper_bound at the
+    very end of the prefix), dyn_index = k itself."""
+    s, W, hdr, addr, val = random_trace(4242, n=2000, n_warps=64)
+    elig = [i for i, x in enumerate(s) if int(x["n_gpr_dst"]) > 0 and not int(x["flags"]) & gen.F_MEM]
+    hdr = hdr.copy()
+    hdr["pc"] = s["pc"][elig[0]]
+    hdr["warp"] = W - 1
+    hdr["active"] = 0x80000000
+    hdr["mask2"] = 0xFFFFFFFF
+    addr = np.zeros((0, 32), np.uint64)
+    val = np.zeros((len(hdr) * int(s["n_gpr_dst"][elig[0]]), 32), np.uint32)
+    so = oracle.sections(oracle.run(s, W, sassi.SASSI_H_INSTCOUNT, hdr, addr, val), len(s), W)
+    assert int(so["counts"][-1]) == len(hdr) and int(so["counts"].sum()) == len(hdr)
+    ctx = sassi.Context(s, W, sassi.SASSI_H_INSTCOUNT)
+    ctx.consume(to_device(s, hdr, addr, val))
+    got = ctx.sample(500, 99)
+    assert np.array_equal(got, oracle.sample(so["counts"], 500, 99))
+    assert (got["thread"] == 32 * W - 1).all()
+    ctx.close()
+
+
 def test_c5_sampled_shards():
     """Config 5 (4x10^9 records over 8 shards of 16,384 warps): each of two shards is generated
     with its global warp ids; a 3x10^6-record prefix of each is exact against the oracle, and the
