@@ -202,7 +202,9 @@ int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
 int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
 
 /* Fold n records (DEVICE buffers) into the context's tables; asynchronous, stream-ordered.
- * Tables accumulate across calls until sassi_reset. Errors: EINVAL, ESTATE (no handler), ECUDA. */
+ * Tables accumulate across calls until sassi_reset. One kernel launch per 2^29 records (the
+ * environment variable SASSI_MAX_LAUNCH_RECORDS, read at sassi_ctx_create, lowers that to a
+ * multiple of SASSI_CHUNK for tests). Errors: EINVAL, ESTATE (no handler), ECUDA. */
 int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, void* stream);
 
 /* Same fold from HOST buffers (pinned or pageable): the library copies slices to the device

@@ -112,6 +112,7 @@ struct sassi_ctx {
   int ctas_per_sm = 0;
   size_t smem_bytes = 0;
   uint64_t launches = 0;
+  uint64_t max_launch = 0;          // records per consume launch (kMaxRecordsPerLaunch unless lowered)
   // host-consume staging (lazily allocated)
   void* stage[2] = {nullptr, nullptr};
   size_t stage_bytes = 0;

@@ -206,6 +206,23 @@ def test_c4_full_instcount_exact_and_sampling():
     ctx.close()
 
 
+def test_multi_launch_split_equals_single_launch(monkeypatch):
+    """sassi_consume splits n records into launches of at most 2^29 (32-bit indices inside a
+    launch). Lowering the split to 4,096 / 65,536 records (SASSI_MAX_LAUNCH_RECORDS) must give the
+    single-launch tables bit for bit on c2 (every handler, payload rows addressed per launch)."""
+    P, mask, d = _gen("c2")
+    S, W = len(d["sites"]), P.total_warps
+    full = gpu_table(d["sites"], W, sassi.SASSI_H_EVERY, d)
+    for per in ("4096", "65536"):
+        monkeypatch.setenv("SASSI_MAX_LAUNCH_RECORDS", per)
+        ctx = sassi.Context(d["sites"], W, sassi.SASSI_H_EVERY)
+        n0 = ctx.kernel_launches()
+        ctx.consume(d)
+        assert ctx.kernel_launches() - n0 == -(-d["n"] // int(per))
+        assert diff_tables(ctx.read_tables(), full, S, W) is None
+        ctx.close()
+
+
 @pytest.mark.parametrize("seed,n,n_warps", [(1, 1, 1), (2, 40, 1), (3, 700, 33), (4, 3000, 300),
                                              (5, 20000, 1500)])
 def test_sampling_edge_cases(seed, n, n_warps):
