@@ -22,7 +22,7 @@ struct NvtxRange {
 
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 constexpr uint32_t EMPTY_KEY = 0xFFFFFFFFu;
-constexpr int kConsumeThreads = 256;          // 8 warps per CTA
+constexpr int kConsumeThreads = 1024;         // 32 warps: one CTA per SM (see DESIGN 6.1)
 constexpr int kWarpsPerCta = kConsumeThreads / 32;
 constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 29;  // 32-bit record / row indices in a launch
 

@@ -203,7 +203,7 @@ uint32_t sm_var_words(uint32_t H) {
 }
 
 template <uint32_t H>
-__global__ void __launch_bounds__(kConsumeThreads, 4) consume_kernel(const ConsumeParams p) {
+__global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
   using Ly = SmLayout<H>;
   constexpr uint32_t kSmDiag = Ly::kDiag, kSmImix = Ly::kImix, kSmH32 = Ly::kH32, kSmH128 = Ly::kH128,
