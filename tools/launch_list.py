@@ -1,5 +1,5 @@
 """Summarise an `ncu --metrics gpu__time_duration.sum --csv` launch list into profiles/ markdown.
-usage: python tools/launch_list.py launches.csv out.md"""
+usage: python tools/launch_list.py launches.csv out.md ["bench command line"]"""
 import collections
 import csv
 import sys
@@ -23,10 +23,11 @@ for d in data:
 tot = sum(v[1] for v in agg.values())
 step = {k: v for k, v in agg.items() if any(s in k for s in STEP)}
 stot = sum(v[1] for v in step.values())
+cmd = sys.argv[3] if len(sys.argv) > 3 else (
+    "python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --no-slowdown --no-injection")
 out = ["# Launch list: `%s`" % sys.argv[1].split("/")[-1], "",
-       "ncu --metrics gpu__time_duration.sum --clock-control none over `python bench.py --steps 2 "
-       "--warmup 1 --no-e2e --no-cpu-baseline --no-slowdown` (generation included). Per-launch times are "
-       "cold-cache and serialised: compare shares, not absolutes.", "",
+       "ncu --metrics gpu__time_duration.sum --clock-control none over `%s` (generation included). "
+       "Per-launch times are cold-cache and serialised: compare shares, not absolutes." % cmd, "",
        "## Kernels of the timed step (reset + consume + sampling)", "",
        "| kernel | launches | total ms | share of step |", "|---|---|---|---|"]
 for k, (n, t) in sorted(step.items(), key=lambda x: -x[1][1]):
