@@ -70,6 +70,7 @@ SIGNATURES = {
     "sassi_ik_trace_copy": (_i, [_vp, _vp, _vp, _vp, _vp]),
     "sassi_ik_output_checksum": (_i, [_vp, ctypes.POINTER(_u64)]),
     "sassi_ik_inject": (_i, [_vp, _vp, _u32, _vp, _vp]),
+    "sassi_ik_trace_fold": (_i, [_vp, _vp, _u32, _u32, _vp, _vp]),
     "sassi_strerror": (ctypes.c_char_p, [_i]),
     "sassi_last_error": (ctypes.c_char_p, []),
 }
@@ -352,6 +353,21 @@ def sassi_ik_output_checksum(ik: int) -> int:
     return c.value
 
 
+SASSI_IK_SERIAL = 1
+TRACE_STATS_DTYPE = np.dtype([("n_records", "<u8"), ("n_addr_rows", "<u8"), ("n_val_rows", "<u8"),
+                              ("max_segment_records", "<u8"), ("ring_bytes", "<u8"),
+                              ("segments", "<u4"), ("blocks_per_segment", "<u4")])
+assert TRACE_STATS_DTYPE.itemsize == 48
+
+
+def sassi_ik_trace_fold(ik: int, ctx: int, blocks_per_segment: int = 0, flags: int = 0,
+                        stream=None) -> dict:
+    st = np.zeros(1, dtype=TRACE_STATS_DTYPE)
+    _check(lib().sassi_ik_trace_fold(ik, ctx, blocks_per_segment, flags, st.ctypes.data,
+                                     _stream(stream)))
+    return {k: int(st[0][k]) for k in TRACE_STATS_DTYPE.names}
+
+
 # error-injection outcomes (include/sassi_ik.h)
 SASSI_INJ_MASKED, SASSI_INJ_SDC, SASSI_INJ_DUE, SASSI_INJ_HANG, SASSI_INJ_NOT_REACHED = range(5)
 INJ_OUTCOME_NAMES = ("masked", "sdc", "due", "hang", "not_reached")
@@ -419,6 +435,13 @@ class InstrumentedKernel:
         torch.cuda.synchronize(dev)
         return dict(hdr=hdr[:n], addr=addr[:na], val=val[:nv], chunk_base=cb, n=n, n_addr_rows=na,
                     n_val_rows=nv, sites=self.sites)
+
+    def trace_fold(self, ctx: Context, blocks_per_segment: int = 0, serial: bool = False,
+                   stream=None) -> dict:
+        """Online trace mode: trace segment by segment into a two-slot ring and fold each segment
+        into ctx on a second stream while the next one is traced."""
+        return sassi_ik_trace_fold(self.handle, ctx.handle, blocks_per_segment,
+                                   SASSI_IK_SERIAL if serial else 0, stream)
 
     def close(self):
         if self.handle:
