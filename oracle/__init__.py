@@ -116,6 +116,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_splitmix64.restype = u64
         L.oracle_select_pcs.argtypes = [u32, u32, vp, u32, vp]
         L.oracle_select_pcs.restype = None
+        L.oracle_dynamic_pcs.argtypes = [vp, u32, vp, u64, vp, u64, vp]
+        L.oracle_dynamic_pcs.restype = u64
         L.oracle_locate_injection.argtypes = [vp, u32, vp, u64, vp, u64, u64, u32, u32, vp]
         L.oracle_locate_injection.restype = ctypes.c_int
         _lib = L
@@ -198,3 +200,18 @@ def locate_injection(sites, hdr, val, thread: int, dyn_index: int, reg_seed: int
     return {"record": int(out[0]), "site": int(out[1]),
             "target": ("gpr", "mem", "pred", "cc")[int(out[2])], "before": int(out[3]),
             "bit": int(out[4])}
+
+
+def dynamic_pcs(sites, hdr):
+    """Insert-on-miss table of the unregistered pcs (Fig.4 l.21-23, DESIGN R25), sorted by pc:
+    -> (uint64 array [n][3] = pc, warp executions, thread executions; records with the reserved
+    pc 0xFFFFFFFF)."""
+    sites = np.ascontiguousarray(sites)
+    hdr = np.ascontiguousarray(hdr)
+    dropped = np.zeros(1, np.uint64)
+    n = lib().oracle_dynamic_pcs(_ptr(sites), len(sites), _ptr(hdr), len(hdr), None, 0,
+                                 _ptr(dropped))
+    out = np.zeros((max(int(n), 1), 3), np.uint64)
+    lib().oracle_dynamic_pcs(_ptr(sites), len(sites), _ptr(hdr), len(hdr), _ptr(out), int(n),
+                             _ptr(dropped))
+    return out[:int(n)], int(dropped[0])
