@@ -395,9 +395,10 @@ def main():
     if not args.no_cpu_baseline and rank == 0 and world == 1:
         cpu = cpu_baseline(args, rec, mask, P)
 
-    slow = None
+    slow = online = None
     if not args.no_slowdown and rank == 0:
         slow = measure_slowdown(dev)
+        online = measure_online_trace(dev, slow)
     inj = None
     if not args.no_injection and rank == 0:
         inj = measure_injection(dev)
@@ -436,6 +437,8 @@ def main():
             line["cpu_baseline"] = cpu
         if slow:
             line["instrumented_slowdown"] = slow
+        if online:
+            line["online_trace"] = online
         if inj:
             line["error_injection"] = inj
         print(json.dumps(line), flush=True)
@@ -505,6 +508,52 @@ def measure_slowdown(dev):
         for k, m in modes.items():
             r[k] = timed(m) / base
         out[name] = r
+        ctx.close()
+        ik.close()
+    return out
+
+
+# online-trace sizes: the timing sizes, except SGEMM at 1024 (2048's trace is ~1.2e9 records)
+ONLINE_SIZES = {"vecadd": 0, "bfs": 0, "sgemm": 1024, "stencil": 0}
+
+
+def measure_online_trace(dev, slow=None):
+    """The trace-driven alternative to inline handlers (L747): each kernel traced
+    segment by segment into a two-slot ring while the previous segment is folded by the consume
+    kernel on a second stream (sassi_ik_trace_fold), all five handlers. Median of 3 (CUDA events on
+    the caller's stream around the blocking call); K = t / t_uninstrumented of the same size;
+    `serial_ms` = the same with the overlap disabled."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    out = {}
+    stream = torch.cuda.current_stream(dev)
+    for name, size in ONLINE_SIZES.items():
+        ik = sassi.InstrumentedKernel(name, size, device=dev.index)
+        ctx = ik.context(sassi.SASSI_H_EVERY)
+
+        def timed(fn, reps=4):
+            ts = []
+            for rep in range(reps):
+                ctx.reset(stream)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                r = fn()
+                b.record(stream)
+                b.synchronize()
+                if rep:
+                    ts.append(a.elapsed_time(b))
+            return statistics.median(ts), r
+
+        base, _ = timed(lambda: ik.run(sassi.SASSI_IK_NONE, None, stream), 6)
+        t_on, st = timed(lambda: ik.trace_fold(ctx, stream=stream))
+        t_ser, _ = timed(lambda: ik.trace_fold(ctx, serial=True, stream=stream))
+        traced = 16 * st["n_records"] + 256 * st["n_addr_rows"] + 128 * st["n_val_rows"]
+        out[name] = {"size": size or "timing", "base_ms": base, "online_ms": t_on, "serial_ms": t_ser,
+                     "K_online": t_on / base, "records": st["n_records"],
+                     "records_per_s": st["n_records"] / (t_on * 1e-3), "trace_bytes": traced,
+                     "segments": st["segments"], "ring_bytes": st["ring_bytes"]}
+        if slow and name in slow and not size:
+            out[name]["K_inline_every"] = slow[name]["every"]
         ctx.close()
         ik.close()
     return out

@@ -201,6 +201,32 @@ int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
  * Errors: EINVAL (unknown pc, not a GLOBAL memory site, k too large), ESTATE, ENOSPC. */
 int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
 
+/* Dynamic sites: Fig.4 l.21-23 (L239) "Find the instruction's counters in a
+ * hash table based on its address. Create a new entry if one does not exist." With this enabled,
+ * every record whose pc is NOT registered (still counted in diag n_unknown_pc; it carries no rows)
+ * also updates an insert-on-miss device hash table keyed by pc: the entry is created on first
+ * sight (CAS, linear probing) and counts warp executions (records) and thread executions
+ * (popc(active); inactive records add a warp execution and no thread). capacity = the number of
+ * distinct unregistered pcs the table must hold (slots: a power of two >= 2 * capacity, >= 32;
+ * capacity 0 disables it). Records that find the table full, or carry the reserved pc
+ * 0xFFFFFFFF, are counted as dropped; results are exact (order-independent) while no record is
+ * dropped. Like sassi_attach_handler: only before the first consume or right after sassi_reset;
+ * sassi_reset clears the table; sassi_merge merges it (capacity is part of the checksum ranks
+ * compare). Errors: EINVAL (capacity > 2^24), ESTATE, ECUDA. DESIGN.md reading R25. */
+int sassi_enable_dynamic_pcs(struct sassi_ctx* ctx, uint32_t capacity);
+
+typedef struct sassi_dyn_pc {
+  uint32_t pc, reserved;
+  uint64_t warp_execs, thread_execs;
+} sassi_dyn_pc;        /* 24 B */
+
+/* Read the dynamic table sorted by pc (canonical: slots depend on insertion order) into HOST
+ * host_out[cap_out]; *n_out = the number of entries (only min(n, cap_out) are written; host_out may
+ * be NULL when cap_out is 0); *n_dropped (may be NULL) = dropped records. Synchronises `stream`.
+ * Errors: EINVAL, ESTATE (not enabled), ECUDA. */
+int sassi_read_dynamic_pcs(struct sassi_ctx* ctx, sassi_dyn_pc* host_out, uint32_t cap_out,
+                           uint32_t* n_out, uint64_t* n_dropped, void* stream);
+
 /* Fold n records (DEVICE buffers) into the context's tables; asynchronous, stream-ordered.
  * Tables accumulate across calls until sassi_reset. One kernel launch per 2^29 records (the
  * environment variable SASSI_MAX_LAUNCH_RECORDS, read at sassi_ctx_create, lowers that to a
@@ -245,7 +271,9 @@ int sassi_sample_sites_device(struct sassi_ctx* ctx, uint32_t k, uint64_t seed,
                               sassi_inj_site* dev_out, uint32_t* dev_status, void* stream);
 
 /* Multi-GPU: merge the tables of all ranks of `nccl_comm` (ncclComm_t) in place with one
- * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits).
+ * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits); with
+ * dynamic pcs enabled, also an ncclAllGather of every rank's dynamic table, which each rank
+ * re-inserts into a cleared table (every rank then holds the same entries).
  * Collective: every rank must call it. Errors: ENCCL, EMISMATCH (site tables differ). */
 int sassi_merge(struct sassi_ctx* ctx, void* nccl_comm, void* stream);
 

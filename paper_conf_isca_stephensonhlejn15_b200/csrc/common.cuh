@@ -76,7 +76,40 @@ struct ConsumeParams {
   uint64_t* table;                  // device table image
   Offsets off;
   uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
+  uint32_t* dyn_keys;               // insert-on-miss table of unregistered pcs (0: disabled) ...
+  unsigned long long* dyn_vals;     // ... [cap][2] warp / thread executions, then dropped records
+  uint32_t dyn_cap, dyn_lg;         // slots (power of two) and log2
 };
+
+// home slot of an unregistered pc in the dynamic table (Fibonacci hashing: dense pcs spread)
+__host__ __device__ __forceinline__ uint32_t dyn_slot(uint32_t pc, uint32_t lg) {
+  return (pc * 0x9E3779B1u) >> (32u - lg);
+}
+
+// Fig.4 l.21-23 "Create a new entry if one does not exist" for an unregistered pc: claim its slot
+// with a CAS (linear probing), then add the counts; a full table (or the reserved pc) counts the
+// records as dropped. (Not inlined: the consume kernel calls it only on the rare miss path.)
+static __device__ __forceinline__ void dyn_insert(uint32_t pc, uint64_t nrec, uint64_t nthr, uint32_t* keys,
+                                        unsigned long long* vals, uint32_t cap, uint32_t lg) {
+  if (pc != EMPTY_KEY) {
+    uint32_t slot = dyn_slot(pc, lg);
+    for (uint32_t probe = 0; probe < cap; ++probe) {
+      uint32_t k = *reinterpret_cast<volatile uint32_t*>(keys + slot);
+      if (k == EMPTY_KEY) {
+        k = atomicCAS(keys + slot, EMPTY_KEY, pc);
+        if (k == EMPTY_KEY) k = pc;
+      }
+      if (k == pc) {
+        atomicAdd(vals + 2 * slot, (unsigned long long)nrec);
+        if (nthr) atomicAdd(vals + 2 * slot + 1, (unsigned long long)nthr);
+        return;
+      }
+      slot = (slot + 1) & (cap - 1);
+    }
+  }
+  atomicAdd(vals + 2 * cap, (unsigned long long)nrec);  // reserved pc or a full table: dropped
+}
+
 
 }  // namespace sassi
 
@@ -122,6 +155,12 @@ struct sassi_ctx {
   // merge scratch
   uint64_t* d_pack = nullptr;
   uint64_t pack_words = 0;
+  // dynamic sites: insert-on-miss table of unregistered pcs (sassi_enable_dynamic_pcs)
+  uint32_t dyn_cap = 0, dyn_lg = 0;
+  uint32_t* d_dyn_keys = nullptr;           // [dyn_cap]
+  unsigned long long* d_dyn_vals = nullptr; // [2 dyn_cap + 1]
+  void* d_dyn_gather = nullptr;             // merge: all ranks' keys and values
+  size_t dyn_gather_bytes = 0;
 };
 
 namespace sassi {
@@ -148,5 +187,6 @@ int launch_sample_device(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site
                          uint32_t* dev_status, cudaStream_t s);
 int launch_merge(sassi_ctx* c, void* comm, cudaStream_t s);
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes);
+int launch_dyn_reset(sassi_ctx* c, cudaStream_t s);
 
 }  // namespace sassi

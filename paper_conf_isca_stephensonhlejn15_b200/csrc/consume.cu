@@ -202,7 +202,9 @@ uint32_t sm_var_words(uint32_t H) {
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
 }
 
-template <uint32_t H>
+// kDyn: the insert-on-miss table of unregistered pcs is enabled (a separate instantiation, so the
+// registered-only kernels carry none of its code)
+template <uint32_t H, bool kDyn>
 __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
   using Ly = SmLayout<H>;
@@ -272,6 +274,19 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     known = valid && e.x == h.x && h.x != EMPTY_KEY;
     c_unk += valid && !known;
     c_inv += known && h.z == 0;
+    if (kDyn) {  // dynamic sites: one insert per distinct unregistered pc of the batch
+      const bool unk = valid && !known;
+      uint32_t um = __ballot_sync(FULL, unk);
+      while (um) {
+        const uint32_t l0 = __ffs(um) - 1;
+        const uint32_t pc0 = __shfl_sync(FULL, h.x, l0);
+        const bool mine = unk && h.x == pc0;
+        const uint32_t g = __ballot_sync(FULL, mine);
+        const uint32_t thr = __reduce_add_sync(FULL, mine ? (uint32_t)__popc(h.z) : 0u);
+        if (lane == l0) dyn_insert(pc0, __popc(g), thr, p.dyn_keys, p.dyn_vals, p.dyn_cap, p.dyn_lg);
+        um &= ~g;
+      }
+    }
     return e;
   };
   // ---- the handlers that read only the header: branch (Fig.4), instruction mix (Fig.3),
@@ -653,27 +668,42 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   }
 }
 
+__global__ void dyn_reset_kernel(uint32_t* keys, unsigned long long* vals, uint32_t cap) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i <= 2 * cap; i += gridDim.x * blockDim.x) {
+    if (i < cap) keys[i] = EMPTY_KEY;
+    vals[i] = 0;
+  }
+}
+
 using KernelFn = void (*)(const ConsumeParams);
 
-template <uint32_t H>
+template <uint32_t H, bool kDyn>
 KernelFn kernel_for() {
-  return consume_kernel<H>;
+  return consume_kernel<H, kDyn>;
 }
 
 template <uint32_t... Hs>
-KernelFn pick(uint32_t mask, std::integer_sequence<uint32_t, Hs...>) {
+KernelFn pick(uint32_t mask, bool dyn, std::integer_sequence<uint32_t, Hs...>) {
   KernelFn fn = nullptr;
-  ((mask == Hs + 1 ? (fn = kernel_for<Hs + 1>(), 0) : 0), ...);
+  ((mask == Hs + 1 ? (fn = dyn ? kernel_for<Hs + 1, true>() : kernel_for<Hs + 1, false>(), 0) : 0), ...);
   return fn;
 }
 
-// one instantiation per non-empty handler set (1..31)
-KernelFn select_kernel(uint32_t mask) {
+// one instantiation per non-empty handler set (1..31), with and without the dynamic-pc table
+KernelFn select_kernel(uint32_t mask, bool dyn) {
   if (mask == 0 || mask > SASSI_H_EVERY) return nullptr;
-  return pick(mask, std::make_integer_sequence<uint32_t, SASSI_H_EVERY>{});
+  return pick(mask, dyn, std::make_integer_sequence<uint32_t, SASSI_H_EVERY>{});
 }
 
 }  // namespace
+
+int launch_dyn_reset(sassi_ctx* c, cudaStream_t s) {
+  if (!c->dyn_cap) return SASSI_OK;
+  dyn_reset_kernel<<<(2 * c->dyn_cap + 256) / 256, 256, 0, s>>>(c->d_dyn_keys, c->d_dyn_vals, c->dyn_cap);
+  SASSI_CUDA(cudaGetLastError());
+  c->launches += 1;
+  return SASSI_OK;
+}
 
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   const uint32_t H = c->mask;
@@ -687,7 +717,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
 }
 
 int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
-  KernelFn fn = select_kernel(c->mask);
+  KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0);
   if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
   SASSI_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->smem_bytes));
   int per_sm = 0;

@@ -20,7 +20,7 @@ typedef struct {
   char internal[128];
 } ncclUniqueId;
 typedef int ncclResult_t;
-enum { kNcclUint64 = 5 };
+enum { kNcclUint32 = 3, kNcclUint64 = 5 };
 enum { kNcclSum = 0, kNcclMax = 2 };
 
 struct Nccl {
@@ -29,6 +29,7 @@ struct Nccl {
   ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
   ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;
   ncclResult_t (*AllReduce)(const void*, void*, size_t, int, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, int, ncclComm_t, cudaStream_t) = nullptr;
   const char* (*GetErrorString)(ncclResult_t) = nullptr;
   bool ok = false;
   std::string why;
@@ -58,9 +59,10 @@ Nccl& nccl() {
     n.CommDestroy = (decltype(n.CommDestroy))dlsym(h, "ncclCommDestroy");
     n.CommCount = (decltype(n.CommCount))dlsym(h, "ncclCommCount");
     n.AllReduce = (decltype(n.AllReduce))dlsym(h, "ncclAllReduce");
+    n.AllGather = (decltype(n.AllGather))dlsym(h, "ncclAllGather");
     n.GetErrorString = (decltype(n.GetErrorString))dlsym(h, "ncclGetErrorString");
     n.ok = n.GetUniqueId && n.CommInitRank && n.CommDestroy && n.CommCount && n.AllReduce &&
-           n.GetErrorString;
+           n.AllGather && n.GetErrorString;
     if (!n.ok) n.why = "libnccl.so.2 lacks an expected symbol";
   });
   return n;
@@ -132,6 +134,21 @@ __global__ void unpack_kernel(uint64_t* __restrict__ t, Offsets o, PackLayout L,
   }
 }
 
+// dynamic tables: every rank's (keys, values) gathered; re-insert all of them into the cleared
+// local table (one thread per gathered slot), dropped records summed
+__global__ void dyn_absorb_kernel(const uint32_t* __restrict__ gk, const unsigned long long* __restrict__ gv,
+                                  uint32_t cap, uint32_t nranks, uint32_t* keys, unsigned long long* vals,
+                                  uint32_t lg) {
+  const uint64_t n = (uint64_t)cap * nranks;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t r = (uint32_t)(i / cap), slot = (uint32_t)(i % cap);
+    const unsigned long long* v = gv + (2ull * cap + 1) * r;
+    if (slot == 0 && v[2ull * cap]) atomicAdd(vals + 2ull * cap, v[2ull * cap]);
+    const uint32_t k = gk[i];
+    if (k != EMPTY_KEY) dyn_insert(k, v[2ull * slot], v[2ull * slot + 1], keys, vals, cap, lg);
+  }
+}
+
 }  // namespace
 
 int launch_merge(sassi_ctx* c, void* comm_v, cudaStream_t s) {
@@ -170,6 +187,32 @@ int launch_merge(sassi_ctx* c, void* comm_v, cudaStream_t s) {
   unpack_kernel<<<grid, 256, 0, s>>>(c->d_table, c->off, L, c->d_pack, (uint32_t)nranks);
   SASSI_CUDA(cudaGetLastError());
   c->launches += 2;
+  // 3) dynamic pcs: slots differ across ranks (insertion order), so gather whole tables and rebuild
+  if (c->dyn_cap) {
+    const uint64_t cap = c->dyn_cap, kb = 4 * cap * nranks, vb = 8 * (2 * cap + 1) * nranks;
+    const size_t need = ((kb + 255) & ~255ull) + vb;
+    if (need > c->dyn_gather_bytes) {
+      cudaFree(c->d_dyn_gather);
+      c->d_dyn_gather = nullptr;
+      c->dyn_gather_bytes = 0;
+      SASSI_CUDA(cudaMalloc(&c->d_dyn_gather, need));
+      c->dyn_gather_bytes = need;
+    }
+    uint32_t* gk = static_cast<uint32_t*>(c->d_dyn_gather);
+    unsigned long long* gv = reinterpret_cast<unsigned long long*>(static_cast<char*>(c->d_dyn_gather) +
+                                                                   ((kb + 255) & ~255ull));
+    r = N.AllGather(c->d_dyn_keys, gk, cap, kNcclUint32, comm, s);
+    if (r) return nccl_err(r, "ncclAllGather(dynamic keys)");
+    r = N.AllGather(c->d_dyn_vals, gv, 2 * cap + 1, kNcclUint64, comm, s);
+    if (r) return nccl_err(r, "ncclAllGather(dynamic values)");
+    int rc = launch_dyn_reset(c, s);
+    if (rc) return rc;
+    const unsigned g2 = (unsigned)std::min<uint64_t>(4096, (cap * nranks + 255) / 256);
+    dyn_absorb_kernel<<<g2, 256, 0, s>>>(gk, gv, c->dyn_cap, (uint32_t)nranks, c->d_dyn_keys,
+                                         c->d_dyn_vals, c->dyn_lg);
+    SASSI_CUDA(cudaGetLastError());
+    c->launches += 1;
+  }
   return SASSI_OK;
 }
 

@@ -62,6 +62,8 @@ SIGNATURES = {
     "sassi_nccl_comm_create": (_i, [ctypes.POINTER(_vp), _i, _i, _vp, _i]),
     "sassi_nccl_comm_destroy": (_i, [_vp]),
     "sassi_kernel_launches": (_i, [_vp, ctypes.POINTER(_u64)]),
+    "sassi_enable_dynamic_pcs": (_i, [_vp, _u32]),
+    "sassi_read_dynamic_pcs": (_i, [_vp, _vp, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u64), _vp]),
     "sassi_ik_create": (_i, [ctypes.POINTER(_vp), _i, _u32, _u64, _i]),
     "sassi_ik_destroy": (None, [_vp]),
     "sassi_ik_sites": (_i, [_vp, _vp, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32)]),
@@ -237,6 +239,25 @@ def sassi_nccl_comm_destroy(comm: int) -> None:
     _check(lib().sassi_nccl_comm_destroy(comm))
 
 
+DYN_PC_DTYPE = np.dtype([("pc", "<u4"), ("reserved", "<u4"), ("warp_execs", "<u8"),
+                         ("thread_execs", "<u8")])
+assert DYN_PC_DTYPE.itemsize == 24
+
+
+def sassi_enable_dynamic_pcs(ctx: int, capacity: int) -> None:
+    _check(lib().sassi_enable_dynamic_pcs(ctx, capacity))
+
+
+def sassi_read_dynamic_pcs(ctx: int, stream=None):
+    """-> (DYN_PC_DTYPE array sorted by pc, dropped records)."""
+    n, dropped = _u32(), _u64()
+    _check(lib().sassi_read_dynamic_pcs(ctx, None, 0, ctypes.byref(n), None, _stream(stream)))
+    out = np.zeros(n.value, dtype=DYN_PC_DTYPE)
+    _check(lib().sassi_read_dynamic_pcs(ctx, out.ctypes.data if n.value else None, n.value,
+                                        ctypes.byref(n), ctypes.byref(dropped), _stream(stream)))
+    return out[:n.value], dropped.value
+
+
 def sassi_kernel_launches(ctx: int) -> int:
     n = _u64()
     _check(lib().sassi_kernel_launches(ctx, ctypes.byref(n)))
@@ -298,6 +319,13 @@ class Context:
 
     def merge(self, comm: int, stream=None):
         sassi_merge(self.handle, comm, stream)
+
+    def enable_dynamic_pcs(self, capacity: int) -> None:
+        """Insert-on-miss table of unregistered pcs (Fig.4 l.21-23)."""
+        sassi_enable_dynamic_pcs(self.handle, capacity)
+
+    def read_dynamic_pcs(self, stream=None):
+        return sassi_read_dynamic_pcs(self.handle, stream)
 
     def kernel_launches(self) -> int:
         return sassi_kernel_launches(self.handle)
