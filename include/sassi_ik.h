@@ -52,23 +52,29 @@ int sassi_ik_trace_totals(sassi_ik* ik, uint64_t* n_rec, uint64_t* n_addr_rows, 
 int sassi_ik_trace_copy(sassi_ik* ik, sassi_hdr* hdr, uint64_t* addr, uint32_t* val, void* stream);
 
 /* ---- Online trace mode ("SASSI traces driving other tools") ----
- * Run the kernel in trace mode one segment of `blocks_per_segment` thread blocks at a time (0 = a
- * segment whose trace regions take about 1 GiB) and fold every segment's records into ctx's
- * tables while the next segment is traced: the producer (the caller's `stream`) traces the segment
- * into per-warp regions and compacts them into a warp-major SRF1 stream in one of two ring slots;
- * a consumer stream owned by the instance builds the slot's chunk index (sassi_index_records) and
- * runs sassi_consume on it, then frees the slot. Device memory is bounded by the segment size, not
- * by the length of the trace. The result equals sassi_consume over the whole-kernel TRACE stream
- * (and the inline handlers' tables): every table is a fold that does not depend on record order.
+ * Trace the kernel and fold its records into ctx's tables segment by segment, each segment's
+ * fold overlapping the tracing of the next. First a count pass runs the kernel once counting
+ * every warp's records and payload rows (exclusive prefixes over the warps give each warp's place
+ * in the warp-major SRF1 stream). Then, per segment of `blocks_per_segment` thread blocks (0 = at
+ * least 4 segments of about 1 GiB of trace each), the producer (the caller's `stream`) runs the
+ * segment's blocks in trace mode writing every record and row straight into its final place in
+ * one of two ring slots sized for the largest segment; a consumer stream owned by the instance
+ * builds the slot's chunk index (sassi_index_records), runs sassi_consume on it and frees the slot
+ * for the segment after next. The pipeline is enqueued without host round trips. Device memory is
+ * bounded by two segments, not by the length of the trace. The kernel must be deterministic
+ * (the four synthetic kernels are): the trace pass checks its counts against the count pass.
+ * The result equals sassi_consume over the whole-kernel TRACE stream (and the inline handlers'
+ * tables): every table is a fold that does not depend on record order.
  * flags: SASSI_IK_SERIAL disables the overlap (each segment is folded before the next is traced;
  * for measurement). ctx must hold exactly this kernel's sites / warps with handlers attached.
  * Blocking: returns after the last fold (stream synchronised). Errors: EINVAL, ESTATE, ECUDA,
- * EFORMAT (a warp overflowed its trace region). `stats` (may be NULL) receives the totals. */
+ * EFORMAT (the trace pass produced other counts than the count pass). `stats` (may be NULL)
+ * receives the totals. */
 enum { SASSI_IK_SERIAL = 1u };
 typedef struct sassi_ik_trace_stats {
   uint64_t n_records, n_addr_rows, n_val_rows;  /* folded, over all segments                  */
   uint64_t max_segment_records;                 /* the largest segment                        */
-  uint64_t ring_bytes;                          /* device bytes of regions + two ring slots   */
+  uint64_t ring_bytes;                          /* device bytes of the two ring slots + counts */
   uint32_t segments, blocks_per_segment;
 } sassi_ik_trace_stats;                         /* 48 B */
 int sassi_ik_trace_fold(sassi_ik* ik, struct sassi_ctx* ctx, uint32_t blocks_per_segment,

@@ -144,6 +144,8 @@ struct sassi_ctx {
   int num_sms = 0;
   int ctas_per_sm = 0;
   size_t smem_bytes = 0;
+  void* launch_fn = nullptr;        // consume kernel last configured (attribute + occupancy) ...
+  size_t launch_smem = 0;           // ... for this shared-memory size
   uint64_t launches = 0;
   uint64_t max_launch = 0;          // records per consume launch (kMaxRecordsPerLaunch unless lowered)
   // host-consume staging (lazily allocated)

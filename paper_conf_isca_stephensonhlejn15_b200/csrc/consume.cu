@@ -16,6 +16,8 @@
 //                                  category totals are formed at the flush
 // Work split: a warp owns one 256-record chunk at a time (chunk_base gives its row offsets) and walks
 // it in 8 batches of 32 records; row indices inside a batch come from ballot prefix sums.
+#include <mutex>
+#include <unordered_map>
 #include <utility>
 
 #include "common.cuh"
@@ -719,11 +721,26 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
 int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
   KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0);
   if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
-  SASSI_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->smem_bytes));
-  int per_sm = 0;
-  SASSI_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kConsumeThreads, c->smem_bytes));
-  if (per_sm < 1) return set_error(SASSI_ENOSPC, "consume kernel does not fit on an SM");
-  c->ctas_per_sm = per_sm;
+  if ((void*)fn != c->launch_fn || c->smem_bytes != c->launch_smem) {  // configure once per kernel
+    {
+      // the attribute is per function and process-wide: only ever raise it (contexts share kernels)
+      static std::mutex mu;
+      static std::unordered_map<void*, size_t> attr;
+      std::lock_guard<std::mutex> lock(mu);
+      size_t& cur = attr[(void*)fn];
+      if (c->smem_bytes > cur) {
+        SASSI_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->smem_bytes));
+        cur = c->smem_bytes;
+      }
+    }
+    int per_sm = 0;
+    SASSI_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kConsumeThreads, c->smem_bytes));
+    if (per_sm < 1) return set_error(SASSI_ENOSPC, "consume kernel does not fit on an SM");
+    c->ctas_per_sm = per_sm;
+    c->launch_fn = (void*)fn;
+    c->launch_smem = c->smem_bytes;
+  }
+  const int per_sm = c->ctas_per_sm;
   const uint64_t units = ((uint64_t)p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
   uint64_t grid = (uint64_t)c->num_sms * per_sm;
   const uint64_t need = (units + kWarpsPerCta - 1) / kWarpsPerCta;
