@@ -16,32 +16,70 @@ from gpu_helpers import to_device, gpu_table  # noqa: E402
 from test_oracle import random_trace  # noqa: E402
 from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi  # noqa: E402
 
+PART = os.environ.get("SANITIZE_PART", "all")  # all | base | online | dynamic
 s = T0.sites()
 hdr, addr, val = T0.records()
 d = to_device(s, hdr, addr, val)
-for mask in (1, 2, 4, 8, 15, 16, 31):
-    t = gpu_table(s, T0.N_WARPS, mask, d)
-    assert np.array_equal(t, oracle.run(s, T0.N_WARPS, mask, hdr, addr, val)), mask
-s2, W, h2, a2, v2 = random_trace(4321, n=3000)
-t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2))
-assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2))
-t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2), pcs=[int(s2[1]["pc"]), int(s2[7]["pc"])])
-assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2, pcs=[1, 7]))
-P, lim, mask, _ = gen.preset("c1")
-dc = gen.generate_device(P, lim)
-ctx = sassi.Context(dc["sites"], P.total_warps, 31)
-ctx.consume(dc)
-ctx.sample(50, 7)
-ctx.close()
-for name, size in (("vecadd", 12800), ("bfs", 4096), ("sgemm", 32), ("stencil", 64)):
-    ik = sassi.InstrumentedKernel(name, size)
-    ctx = ik.context(sassi.SASSI_H_EVERY)
-    for mode in (0, 1, 2, 4, 8, 16, 15, 31, sassi.SASSI_IK_NULL_ABI):
-        ctx.reset()
-        ik.run(mode, ctx if mode & 31 else None)
-    ik.trace(ctx)
+if PART in ("all", "base"):
+    for mask in (1, 2, 4, 8, 15, 16, 31):
+        t = gpu_table(s, T0.N_WARPS, mask, d)
+        assert np.array_equal(t, oracle.run(s, T0.N_WARPS, mask, hdr, addr, val)), mask
+    s2, W, h2, a2, v2 = random_trace(4321, n=3000)
+    t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2))
+    assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2))
+    t = gpu_table(s2, W, 31, to_device(s2, h2, a2, v2), pcs=[int(s2[1]["pc"]), int(s2[7]["pc"])])
+    assert np.array_equal(t, oracle.run(s2, W, 31, h2, a2, v2, pcs=[1, 7]))
+    P, lim, mask, _ = gen.preset("c1")
+    dc = gen.generate_device(P, lim)
+    ctx = sassi.Context(dc["sites"], P.total_warps, 31)
+    ctx.consume(dc)
+    ctx.sample(50, 7)
     ctx.close()
-    ik.injection_campaign(k=20, seed=3)
-    ik.close()
+    for name, size in (("vecadd", 12800), ("bfs", 4096), ("sgemm", 32), ("stencil", 64)):
+        ik = sassi.InstrumentedKernel(name, size)
+        ctx = ik.context(sassi.SASSI_H_EVERY)
+        for mode in (0, 1, 2, 4, 8, 16, 15, 31, sassi.SASSI_IK_NULL_ABI):
+            ctx.reset()
+            ik.run(mode, ctx if mode & 31 else None)
+        ik.trace(ctx)
+        ctx.close()
+        ik.injection_campaign(k=20, seed=3)
+        ik.close()
+
+if PART in ("all", "online"):
+    # online trace mode (count pass, placed trace into the ring, index + fold on the consumer stream)
+    for name, size in (("vecadd", 1 << 16), ("bfs", 4096), ("sgemm", 64), ("stencil", 64)):
+        ik = sassi.InstrumentedKernel(name, size)
+        ctx = ik.context(sassi.SASSI_H_EVERY)
+        rec = ik.trace(ctx)
+        h = gen.to_host(rec)
+        want = oracle.run(h["sites"], ik.n_warps, 31, h["hdr"], h["addr"], h["val"])
+        for bps, serial in ((0, True), (3, False)):
+            ctx.reset()
+            ik.trace_fold(ctx, blocks_per_segment=bps, serial=serial)
+            assert np.array_equal(ctx.read_tables(), want), (name, bps)
+        ctx.close()
+        ik.close()
+
+if PART in ("all", "dynamic"):
+    # dynamic sites: an empty site table (every record inserted on miss) and a 1-rank merge
+    hs = np.zeros((5000, 4), np.uint32)
+    rng = np.random.default_rng(5)
+    hs[:, 0] = 0x1000 + 16 * rng.integers(0, 300, 5000)
+    hs[:, 2] = rng.integers(0, 2**32, 5000, dtype=np.uint64).astype(np.uint32)
+    hs = hs.view(oracle.HDR_DTYPE).reshape(-1)
+    s0 = np.zeros(0, dtype=oracle.SITE_DTYPE)
+    ctx = sassi.Context(s0, 4, 15)
+    ctx.enable_dynamic_pcs(300)
+    ctx.consume(to_device(s0, hs, None, None))
+    uid = sassi.sassi_nccl_get_unique_id()
+    comm = sassi.sassi_nccl_comm_create(1, 0, uid, 0)
+    ctx.merge(comm)
+    sassi.sassi_nccl_comm_destroy(comm)
+    dyn, dropped = ctx.read_dynamic_pcs()
+    odyn, odrop = oracle.dynamic_pcs(s0, hs)
+    assert [[int(e["pc"]), int(e["warp_execs"]), int(e["thread_execs"])] for e in dyn] == odyn.tolist()
+    ctx.close()
+
 torch.cuda.synchronize()
 print("sanitize workload ok")
