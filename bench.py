@@ -478,11 +478,15 @@ def measure_slowdown(dev):
     """Instrumented-kernel slowdown K = t_instrumented / t_uninstrumented (the K column of the
     paper's Table 3), median of 5 runs each (L679), per handler, for the four synthetic
     kernels at their timing sizes; `null_abi` is the paper's stubbed-handler control (L687);
-    `instmix` is Fig.3's handler (L193-L199), `all` the four case studies, `every` all five."""
+    `instmix` is Fig.3's handler (L193-L199), `all` the four case studies, `every` all five;
+    `*_smem` the same with the opt-in per-CTA shared-memory tables (the default uses none, L741)."""
     import torch
     from paper_conf_isca_stephensonhlejn15_b200 import sassi
     modes = {"null_abi": sassi.SASSI_IK_NULL_ABI, "branch": 1, "memdiv": 2, "value": 4,
              "instcount": 8, "instmix": 16, "all": 15, "every": 31}
+    # the same handlers with the opt-in per-CTA shared-memory tables (SASSI_IK_SMEM)
+    modes.update({k + "_smem": m | sassi.SASSI_IK_SMEM for k, m in list(modes.items())
+                  if 0 < m <= sassi.SASSI_H_EVERY})
     out = {}
     stream = torch.cuda.current_stream(dev)
     for name in ("vecadd", "bfs", "sgemm", "stencil"):

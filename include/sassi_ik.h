@@ -26,7 +26,8 @@ extern "C" {
 #endif
 
 enum { SASSI_IK_VECADD = 0, SASSI_IK_BFS = 1, SASSI_IK_SGEMM = 2, SASSI_IK_STENCIL = 3 };
-enum { SASSI_IK_NONE = 0u, SASSI_IK_TRACE = 64u, SASSI_IK_NULL_ABI = 128u };  /* above SASSI_H_EVERY */
+enum { SASSI_IK_NONE = 0u, SASSI_IK_TRACE = 64u, SASSI_IK_NULL_ABI = 128u,  /* above SASSI_H_EVERY */
+       SASSI_IK_SMEM = 1024u };  /* | a handler mask: opt-in per-CTA shared-memory aggregation */
 
 typedef struct sassi_ik sassi_ik;
 
@@ -39,7 +40,11 @@ void sassi_ik_destroy(sassi_ik* ik);
 int sassi_ik_sites(sassi_ik* ik, sassi_site* out, uint32_t cap, uint32_t* n_sites, uint32_t* n_warps);
 
 /* Run once. mode = SASSI_IK_NONE | SASSI_IK_NULL_ABI | SASSI_IK_TRACE | one of the handler masks
- * above (1, 2, 4, 8, 16, 15, 31; EINVAL otherwise);
+ * above (1, 2, 4, 8, 16, 15, 31; EINVAL otherwise), optionally | SASSI_IK_SMEM. By default the
+ * inline handlers use no shared memory (a handler's use of it can break or slow a kernel that needs
+ * it all): each warp's totals go to global memory at kernel exit. SASSI_IK_SMEM opts
+ * in to per-CTA tables in shared memory (the warps fold into them at exit, one flush per CTA; up
+ * to 14 words per site + 8 KB with memdiv), which is faster for kernels of many short-lived warps;
  * handler bits fold into ctx's tables (ctx must hold exactly this kernel's sites / warps).
  * Asynchronous on `stream` except SASSI_IK_TRACE, which synchronises. */
 int sassi_ik_run(sassi_ik* ik, uint32_t mode, struct sassi_ctx* ctx, void* stream);

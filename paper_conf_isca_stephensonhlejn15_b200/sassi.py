@@ -27,7 +27,7 @@ SASSI_H_BRANCH, SASSI_H_MEMDIV, SASSI_H_VALUE, SASSI_H_INSTCOUNT, SASSI_H_ALL = 
 SASSI_H_INSTMIX, SASSI_H_EVERY = 16, 31
 SASSI_CHUNK = 256
 SASSI_IK_VECADD, SASSI_IK_BFS, SASSI_IK_SGEMM, SASSI_IK_STENCIL = 0, 1, 2, 3
-SASSI_IK_NONE, SASSI_IK_TRACE, SASSI_IK_NULL_ABI = 0, 64, 128
+SASSI_IK_NONE, SASSI_IK_TRACE, SASSI_IK_NULL_ABI, SASSI_IK_SMEM = 0, 64, 128, 1024
 
 # every function declared in include/*.h: name -> (restype, argtypes)
 _vp, _u32, _u64, _i = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int

@@ -39,11 +39,12 @@ def trace_and_fold(ik, mask):
 
 @pytest.mark.parametrize("name", list(SMALL))
 @pytest.mark.parametrize("mask", [sassi.SASSI_H_ALL, sassi.SASSI_H_EVERY])
-def test_inline_equals_trace_fold_equals_oracle(name, mask):
+@pytest.mark.parametrize("smem", [0, sassi.SASSI_IK_SMEM])
+def test_inline_equals_trace_fold_equals_oracle(name, mask, smem):
     ik = sassi.InstrumentedKernel(name, SMALL[name])
     S, W = len(ik.sites), ik.n_warps
     ctx = ik.context(mask)
-    ik.run(mask, ctx)
+    ik.run(mask | smem, ctx)
     t_inline = ctx.read_tables()
     ctx.close()
     rec, t_fold = trace_and_fold(ik, mask)
@@ -58,10 +59,11 @@ def test_inline_equals_trace_fold_equals_oracle(name, mask):
 
 @pytest.mark.parametrize("name", list(SMALL))
 @pytest.mark.parametrize("mask", [1, 2, 4, 8, 16])
-def test_single_handler_inline(name, mask):
+@pytest.mark.parametrize("smem", [0, sassi.SASSI_IK_SMEM])
+def test_single_handler_inline(name, mask, smem):
     ik = sassi.InstrumentedKernel(name, SMALL[name])
     ctx = ik.context(mask)
-    ik.run(mask, ctx)
+    ik.run(mask | smem, ctx)
     t_inline = ctx.read_tables()
     ctx.close()
     _, t_fold = trace_and_fold(ik, mask)
