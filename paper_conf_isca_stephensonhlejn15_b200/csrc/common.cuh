@@ -25,6 +25,8 @@ constexpr uint32_t EMPTY_KEY = 0xFFFFFFFFu;
 constexpr int kConsumeThreads = 1024;         // 32 warps: one CTA per SM (see DESIGN 6.1)
 constexpr int kWarpsPerCta = kConsumeThreads / 32;
 constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 29;  // 32-bit record / row indices in a launch
+constexpr uint32_t kDynLocalLg = 9, kDynLocal = 1u << kDynLocalLg;  // per-CTA dynamic-pc cache slots
+constexpr uint32_t kDynLocalWords = 4 * kDynLocal;                  // key + count (u32) + threads (u64)
 
 // Packed per-site info word in the hash (bit layout). The companion cidx word holds the
 // site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).

@@ -217,7 +217,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
   uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
   uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + (Ly::kVal ? p.nvd : 0u));  // counters
-  uint32_t* s_pcm = s_priv + (p.priv ? kWarpsPerCta : 1u) * p.pw;  // [npcm][32][32] per-PC matrices
+  // [npcm][32][32] per-PC matrices (the private counters exist only for handler sets that count)
+  uint32_t* s_pcm = s_priv + ((H & kCounters) ? (p.priv ? kWarpsPerCta : 1u) * p.pw : 0u);
+  // dynamic sites: a per-CTA insert-on-miss cache of unregistered pcs (keys, record counts, thread
+  // counts), flushed into the global table at CTA exit
+  uint32_t* const s_dkey = s_pcm + 1024 * p.npcm;
+  uint32_t* const s_dcnt = s_dkey + kDynLocal;
+  unsigned long long* const s_dthr = reinterpret_cast<unsigned long long*>(s_dcnt + kDynLocal);
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
 
   const uint32_t tid = threadIdx.x;
@@ -229,6 +235,12 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
   if (H & SASSI_H_MEMDIV)
     for (uint32_t i = tid; i < 1024 * p.npcm; i += blockDim.x) s_pcm[i] = 0;
+  if (kDyn)
+    for (uint32_t i = tid; i < kDynLocal; i += blockDim.x) {
+      s_dkey[i] = EMPTY_KEY;
+      s_dcnt[i] = 0;
+      s_dthr[i] = 0;
+    }
   if (Ly::kVal && tid < kWarpsPerCta) mbar_init(reinterpret_cast<uint64_t*>(sm + kSmBar) + tid, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
@@ -276,17 +288,27 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     known = valid && e.x == h.x && h.x != EMPTY_KEY;
     c_unk += valid && !known;
     c_inv += known && h.z == 0;
-    if (kDyn) {  // dynamic sites: one insert per distinct unregistered pc of the batch
-      const bool unk = valid && !known;
-      uint32_t um = __ballot_sync(FULL, unk);
-      while (um) {
-        const uint32_t l0 = __ffs(um) - 1;
-        const uint32_t pc0 = __shfl_sync(FULL, h.x, l0);
-        const bool mine = unk && h.x == pc0;
-        const uint32_t g = __ballot_sync(FULL, mine);
-        const uint32_t thr = __reduce_add_sync(FULL, mine ? (uint32_t)__popc(h.z) : 0u);
-        if (lane == l0) dyn_insert(pc0, __popc(g), thr, p.dyn_keys, p.dyn_vals, p.dyn_cap, p.dyn_lg);
-        um &= ~g;
+    if (kDyn) {  // dynamic sites: each lane adds its own unregistered record to the CTA's cache
+      if (valid && !known) {
+        bool done = false;
+        if (h.x != EMPTY_KEY) {
+          uint32_t slot = dyn_slot(h.x, kDynLocalLg);
+          for (uint32_t probe = 0; probe < 8 && !done; ++probe) {
+            uint32_t k = *reinterpret_cast<volatile uint32_t*>(s_dkey + slot);
+            if (k == EMPTY_KEY) {
+              k = atomicCAS(s_dkey + slot, EMPTY_KEY, h.x);
+              if (k == EMPTY_KEY) k = h.x;
+            }
+            if (k == h.x) {
+              atomicAdd(s_dcnt + slot, 1u);
+              if (h.z) atomicAdd(s_dthr + slot, (unsigned long long)__popc(h.z));
+              done = true;
+            }
+            slot = (slot + 1) & (kDynLocal - 1);
+          }
+        }
+        // a long probe or the reserved pc: the global table (Fig.4 l.21-23's device-wide table)
+        if (!done) dyn_insert(h.x, 1, (uint32_t)__popc(h.z), p.dyn_keys, p.dyn_vals, p.dyn_cap, p.dyn_lg);
       }
     }
     return e;
@@ -595,6 +617,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
 
   // ---- flush: sum the warps' private counters, fold into the global u64 image ----
   if (tid < 4 && s_diag[tid]) atomicAdd(&table[tid], (unsigned long long)s_diag[tid]);
+  if (kDyn)
+    for (uint32_t i = tid; i < kDynLocal; i += blockDim.x)
+      if (s_dkey[i] != EMPTY_KEY && s_dcnt[i])
+        dyn_insert(s_dkey[i], s_dcnt[i], s_dthr[i], p.dyn_keys, p.dyn_vals, p.dyn_cap, p.dyn_lg);
   auto sum_words = [&](uint32_t off) -> uint4 {
     uint4 t = make_uint4(0, 0, 0, 0);
     for (uint32_t w = 0; w < n_regions; ++w) {
@@ -714,6 +740,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX))
     words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
   if (H & SASSI_H_MEMDIV) words += 1024ull * c->npcm;  // per-PC matrices
+  if (c->dyn_cap) words += kDynLocalWords;              // the CTA's dynamic-pc cache
   *bytes = 4 * words;
   return 0;
 }
