@@ -147,3 +147,35 @@ def test_merge_single_rank_nccl_rebuilds_dynamic_table():
     assert np.array_equal(after, before)
     odyn, odrop = oracle.dynamic_pcs(s2, hdr)
     assert as_list(dyn) == odyn.tolist() and dropped == odrop
+
+
+@pytest.mark.parametrize("mask", [sassi.SASSI_H_INSTCOUNT, sassi.SASSI_H_BRANCH | sassi.SASSI_H_INSTMIX])
+def test_c4_prefix_half_the_sites_unregistered(mask):
+    """The error-injection profiling stream (c4) at scale: its first 10^7 records with every other
+    site unregistered, under header-only handler sets (rows are never read, so the stream stays
+    valid). The registered-site tables and the dynamic table both equal the oracle's."""
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
+    P, lim, _, _ = gen.preset("c4")
+    d = gen.generate_device(P, 10_000_000)
+    s_all = d["sites"]
+    s2 = s_all[::2].copy()
+    W = P.total_warps
+    hdr = d["hdr"][: d["n"]].cpu().numpy().view(np.uint32).reshape(-1, 4).view(oracle.HDR_DTYPE).reshape(-1)
+    rec = dict(hdr=d["hdr"], addr=d["addr"][:0], val=d["val"][:0], chunk_base=d["chunk_base"],
+               n=d["n"], n_addr_rows=0, n_val_rows=0)
+    t, dyn, dropped = fold(s2, W, mask, rec, len(s_all))
+    # header-only handlers read no rows (c4 is generated without them): the oracle gets the row
+    # counts its registered sites imply (SRF1) and never dereferences a row
+    order = np.argsort(s2["pc"])
+    pos = np.searchsorted(s2["pc"][order], hdr["pc"])
+    pos = np.minimum(pos, len(s2) - 1)
+    idx = order[pos]
+    reg = s2["pc"][idx] == hdr["pc"]
+    na = int(((s2["flags"][idx] & oracle.F_MEM) != 0)[reg].sum())
+    nv = int(s2["n_gpr_dst"][idx][reg].astype(np.int64).sum())
+    o = oracle.consume(oracle.table_init(len(s2), W, mask), s2, W, mask, hdr, None, None,
+                       n_addr_rows=na, n_val_rows=nv)
+    assert diff_tables(t, o, len(s2), W) is None
+    odyn, odrop = oracle.dynamic_pcs(s2, hdr)
+    assert dyn == odyn.tolist() and dropped == odrop == 0
+    assert len(dyn) == len(s_all) - len(s2)
