@@ -67,16 +67,24 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x, uint32_t lane) {
   return x;
 }
 
-// Bitonic sort of one key per lane across the warp (ascending in lane order).
+// Bitonic sort of one key per lane across the warp (ascending in lane order), in the "flip" form:
+// each merge of blocks of k starts by comparing lane i with lane i ^ (k - 1) (the reversed partner)
+// and continues with i ^ j; in every step the lower lane of a pair keeps the minimum, so a lane's
+// direction is one of its five index bits (no per-step direction arithmetic: 2 ALU ops a step).
 template <typename T>
 __device__ __forceinline__ T warp_sort(T v, uint32_t lane) {
 #pragma unroll
   for (uint32_t k = 2; k <= 32; k <<= 1) {
+    {
+      const T o = __shfl_xor_sync(FULL, v, k - 1);
+      const bool lower = (lane & (k >> 1)) == 0;
+      v = lower ? (o < v ? o : v) : (o > v ? o : v);
+    }
 #pragma unroll
-    for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+    for (uint32_t j = k >> 2; j > 0; j >>= 1) {
       const T o = __shfl_xor_sync(FULL, v, j);
-      const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0);
-      v = keep_min ? (o < v ? o : v) : (o > v ? o : v);
+      const bool lower = (lane & j) == 0;
+      v = lower ? (o < v ? o : v) : (o > v ? o : v);
     }
   }
   return v;
