@@ -91,6 +91,11 @@
 extern "C" {
 #endif
 
+/* Opaque context (one per device; owns the device tables and the site hash). Declared here so
+ * the prototypes below all name the same type in C as well as in C++. */
+struct sassi_ctx;
+typedef struct sassi_ctx sassi_ctx;
+
 #define SASSI_ABI_VERSION 3u
 #define SASSI_WARP_SIZE 32u
 #define SASSI_CHUNK 256u           /* records per chunk_base entry */
