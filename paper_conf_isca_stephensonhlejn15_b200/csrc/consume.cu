@@ -270,13 +270,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   // Only for handler sets without payload rows: with them, the 4 extra registers cost more than
   // the transposes they save (measured: c3 2.90 -> 3.06 ms)
   constexpr bool kVertical = !(H & (SASSI_H_MEMDIV | SASSI_H_VALUE));
-  uint32_t vp0 = 0, vp1 = 0, vp2 = 0, vp3 = 0, vn = 0;
+  // (flushed every 5 iterations of the 3-batch header loop, and whenever the accumulator moves)
+  uint32_t vp0 = 0, vp1 = 0, vp2 = 0, vp3 = 0;
   auto flush_planes = [&]() {
-    if (vn) {
+    if (__any_sync(FULL, (vp0 | vp1 | vp2 | vp3) != 0)) {
       acc += __popc(transpose32<true>(vp0, lane)) + 2 * __popc(transpose32<true>(vp1, lane)) +
              4 * __popc(transpose32<true>(vp2, lane)) + 8 * __popc(transpose32<true>(vp3, lane));
       vp0 = vp1 = vp2 = vp3 = 0;
-      vn = 0;
     }
   };
   uint32_t err = 0;
@@ -340,15 +340,18 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
     if (H & SASSI_H_INSTCOUNT) {
       uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
-      if (E != 0 && h.y >= p.n_warps) {
-        ++c_bad;
-        E = 0;
-      }
+      auto drop_bad_warps = [&]() {  // records of warps outside the counts (n_bad_warp)
+        if (E != 0 && h.y >= p.n_warps) {
+          ++c_bad;
+          E = 0;
+        }
+      };
       uint32_t pend;
       if (kVertical) {
         // the usual case in a warp-major stream: every eligible lane is on the accumulator's trace
-        // warp -> add E into the vertical counters (one vote decides it)
-        if (!__any_sync(FULL, E != 0 && h.y != acc_w)) {
+        // warp (a checked one: acc_w != FULL) -> add E into the vertical counters; one vote decides
+        // it, and only the other path needs the warp-range check
+        if (acc_w != FULL && !__any_sync(FULL, E != 0 && h.y != acc_w)) {
           const uint32_t k0 = vp0 & E;
           vp0 ^= E;
           const uint32_t k1 = vp1 & k0;
@@ -356,13 +359,14 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
           const uint32_t k2 = vp2 & k1;
           vp2 ^= k1;
           vp3 ^= k2;  // at most 15 additions between flushes: no carry out of plane 3
-          if (++vn == 15) flush_planes();
           pend = 0;
         } else {
+          drop_bad_warps();
           flush_planes();
           pend = __ballot_sync(FULL, E != 0);
         }
       } else {
+        drop_bad_warps();
         pend = __ballot_sync(FULL, E != 0);
       }
       while (pend) {
@@ -398,7 +402,12 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     uint4 q[kDepth];
 #pragma unroll
     for (uint32_t k = 0; k < kDepth; ++k) q[k] = hload(first_rec(k));
+    uint32_t it = 0;  // iterations since the vertical counters were last folded
     for (uint32_t t = 0;; t += kDepth) {
+      if ((H & SASSI_H_INSTCOUNT) && kVertical && ++it == 6) {  // <= 15 additions between folds
+        flush_planes();
+        it = 1;
+      }
       bool done = false;
 #pragma unroll
       for (uint32_t k = 0; k < kDepth; ++k) {
