@@ -282,6 +282,25 @@ int sassi_sample_sites_device(struct sassi_ctx* ctx, uint32_t k, uint64_t seed,
  * Collective: every rank must call it. Errors: ENCCL, EMISMATCH (site tables differ). */
 int sassi_merge(struct sassi_ctx* ctx, void* nccl_comm, void* stream);
 
+/* ---- Fused fold + merge over peer memory (one node: NVLink / NVSwitch P2P, or one device) ----
+ * Instead of folding and then running sassi_merge's collective, every rank can fold straight into
+ * every rank's table image: each rank exports its image (a CUDA IPC handle of SASSI_IPC_HANDLE_BYTES
+ * bytes, exchanged by the caller, e.g. torch.distributed.all_gather_object) and opens the others'
+ * with sassi_add_peer_table. From then on every table update of sassi_consume (the CTA-exit flush
+ * and the per-thread count adds) is also applied, as an atomic over NVLink, to each peer's image:
+ * sums add and the AND masks AND (PAPER.md's tables are commutative folds), so once every rank's
+ * folds have completed every image holds the merged tables — sassi_merge's result without a
+ * collective. Protocol: sassi_reset on every rank, a barrier, the folds, a barrier (each after a
+ * stream synchronise), then sassi_read_tables anywhere. The dynamic-pc table and the inline
+ * handlers of sassi_ik_run are not included (use sassi_merge for those).
+ * sassi_add_peer_table: only before the first consume or right after sassi_reset; the peer's image
+ * must have this context's layout (EMISMATCH otherwise); at most 7 peers (ENOSPC).
+ * sassi_clear_peer_tables synchronises the device and closes the handles. */
+#define SASSI_IPC_HANDLE_BYTES 64
+int sassi_ipc_table_handle(struct sassi_ctx* ctx, void* handle_out);
+int sassi_add_peer_table(struct sassi_ctx* ctx, const void* handle);
+int sassi_clear_peer_tables(struct sassi_ctx* ctx);
+
 /* NCCL bootstrap helpers (NCCL is loaded lazily with dlopen; only sassi_merge needs it). */
 int sassi_nccl_get_unique_id(void* out_128_bytes);
 int sassi_nccl_comm_create(void** comm_out, int nranks, int rank, const void* unique_id_128_bytes,

@@ -27,6 +27,7 @@ constexpr int kWarpsPerCta = kConsumeThreads / 32;
 constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 29;  // 32-bit record / row indices in a launch
 constexpr uint32_t kDynLocalLg = 9, kDynLocal = 1u << kDynLocalLg;  // per-CTA dynamic-pc cache slots
 constexpr uint32_t kDynLocalWords = 4 * kDynLocal;                  // key + count (u32) + threads (u64)
+constexpr uint32_t kMaxPeers = 7;   // fused merge over peer memory: up to 8 GPUs of one node
 
 // Packed per-site info word in the hash (bit layout). The companion cidx word holds the
 // site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).
@@ -81,6 +82,8 @@ struct ConsumeParams {
   uint32_t* dyn_keys;               // insert-on-miss table of unregistered pcs (0: disabled) ...
   unsigned long long* dyn_vals;     // ... [cap][2] warp / thread executions, then dropped records
   uint32_t dyn_cap, dyn_lg;         // slots (power of two) and log2
+  unsigned long long* peers[kMaxPeers];  // fused merge: peers' table images (same layout) ...
+  uint32_t n_peers;                 // ... that every flush atomic also goes to
 };
 
 // home slot of an unregistered pc in the dynamic table (Fibonacci hashing: dense pcs spread)
@@ -165,6 +168,9 @@ struct sassi_ctx {
   unsigned long long* d_dyn_vals = nullptr; // [2 dyn_cap + 1]
   void* d_dyn_gather = nullptr;             // merge: all ranks' keys and values
   size_t dyn_gather_bytes = 0;
+  // fused merge over peer memory: peers' table images opened from CUDA IPC handles
+  unsigned long long* peer_tables[sassi::kMaxPeers] = {};
+  uint32_t n_peers = 0;
 };
 
 namespace sassi {

@@ -281,6 +281,16 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   };
   uint32_t err = 0;
   unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
+  // every table update goes to this context's image and to the peers' (fused merge: the atomics
+  // travel over NVLink to the other GPUs' images, so no collective runs after the fold)
+  auto gadd = [&](uint64_t off, unsigned long long v) {
+    atomicAdd(table + off, v);
+    for (uint32_t j = 0; j < p.n_peers; ++j) atomicAdd(p.peers[j] + off, v);
+  };
+  auto gand = [&](uint64_t off, unsigned long long v) {
+    atomicAnd(table + off, v);
+    for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd(p.peers[j] + off, v);
+  };
 
   // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239). Returns the
   // slot {key, info, cidx, site}; `known` = a registered site (0xFFFFFFFF is never registered) ----
@@ -375,7 +385,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
         const uint32_t cnt = __popc(transpose32<kVertical>(mine ? E : 0u, lane));
         if (w0 != acc_w) {
           if (acc_w != FULL && acc)
-            atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+            gadd(p.off.counts + 32ull * acc_w + lane, (unsigned long long)acc);
           acc_w = w0;
           acc = 0;
         }
@@ -614,7 +624,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   }
   if (H & SASSI_H_INSTCOUNT) {
     if (kVertical) flush_planes();
-    if (acc_w != FULL && acc) atomicAdd(&table[p.off.counts + 32ull * acc_w + lane], (unsigned long long)acc);
+    if (acc_w != FULL && acc) gadd(p.off.counts + 32ull * acc_w + lane, (unsigned long long)acc);
   }
   // ---- diagnostics: warp-reduce, one smem atomic per warp ----
   uint32_t* const s_diag = sm + kSmDiag;
@@ -633,7 +643,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   __syncthreads();
 
   // ---- flush: sum the warps' private counters, fold into the global u64 image ----
-  if (tid < 4 && s_diag[tid]) atomicAdd(&table[tid], (unsigned long long)s_diag[tid]);
+  if (tid < 4 && s_diag[tid]) gadd(tid, (unsigned long long)s_diag[tid]);
   if (kDyn)
     for (uint32_t i = tid; i < kDynLocal; i += blockDim.x)
       if (s_dkey[i] != EMPTY_KEY && s_dcnt[i])
@@ -653,30 +663,30 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     for (uint32_t bi = tid; bi < p.nb; bi += blockDim.x) {
       const uint4 t = sum_words(4 * bi);
       if (t.x == 0) continue;
-      unsigned long long* g = table + p.off.br + 5ull * p.flush_b[bi];
-      atomicAdd(g + 0, (unsigned long long)t.x);
-      atomicAdd(g + 1, (unsigned long long)t.y);
-      if (t.z) atomicAdd(g + 2, (unsigned long long)t.z);
-      if (t.y - t.z) atomicAdd(g + 3, (unsigned long long)(t.y - t.z));  // not taken = active - taken
-      if (t.w) atomicAdd(g + 4, (unsigned long long)t.w);
+      const uint64_t g = p.off.br + 5ull * p.flush_b[bi];
+      gadd(g + 0, (unsigned long long)t.x);
+      gadd(g + 1, (unsigned long long)t.y);
+      if (t.z) gadd(g + 2, (unsigned long long)t.z);
+      if (t.y - t.z) gadd(g + 3, (unsigned long long)(t.y - t.z));  // not taken = active - taken
+      if (t.w) gadd(g + 4, (unsigned long long)t.w);
     }
   }
   if (H & SASSI_H_MEMDIV) {
     for (uint32_t m = tid; m < p.nm; m += blockDim.x) {
       const uint4 t = sum_words(PB + 4 * m);
       if (t.x == 0) continue;
-      unsigned long long* g = table + p.off.mem + 4ull * p.flush_m[m];
-      atomicAdd(g + 0, (unsigned long long)t.x);
-      atomicAdd(g + 1, (unsigned long long)t.y);
-      atomicAdd(g + 2, (unsigned long long)t.z);
-      atomicAdd(g + 3, (unsigned long long)t.w);
+      const uint64_t g = p.off.mem + 4ull * p.flush_m[m];
+      gadd(g + 0, (unsigned long long)t.x);
+      gadd(g + 1, (unsigned long long)t.y);
+      gadd(g + 2, (unsigned long long)t.z);
+      gadd(g + 3, (unsigned long long)t.w);
     }
     for (uint32_t c = tid; c < 2048; c += blockDim.x) {
       const uint32_t v = sm[kSmH32 + c];
-      if (v) atomicAdd(table + (c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024)), (unsigned long long)v);
+      if (v) gadd(c < 1024 ? p.off.h32 + c : p.off.h128 + (c - 1024), (unsigned long long)v);
     }
     for (uint32_t c = tid; c < 1024 * p.npcm; c += blockDim.x)
-      if (s_pcm[c]) atomicAdd(table + p.off.pcmat + c, (unsigned long long)s_pcm[c]);
+      if (s_pcm[c]) gadd(p.off.pcmat + c, (unsigned long long)s_pcm[c]);
   }
   if (H & SASSI_H_INSTMIX) {
     unsigned long long* const s_imix = reinterpret_cast<unsigned long long*>(sm + kSmImix);
@@ -684,13 +694,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       uint32_t t = 0;
       for (uint32_t w = 0; w < n_regions; ++w) t += s_priv[w * p.pw + p.px + st];
       if (t == 0) continue;
-      atomicAdd(table + p.off.mix + st, (unsigned long long)t);
+      gadd(p.off.mix + st, (unsigned long long)t);
       const uint32_t cat = p.flush_x[st];
       for (uint32_t k = 0; k < 7; ++k)
         if ((cat >> k) & 1u) atomicAdd(s_imix + k, (unsigned long long)t);
     }
     __syncthreads();
-    if (tid < 7 && s_imix[tid]) atomicAdd(table + p.off.imix + tid, s_imix[tid]);
+    if (tid < 7 && s_imix[tid]) gadd(p.off.imix + tid, s_imix[tid]);
   }
   if (H & SASSI_H_VALUE) {
     for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
@@ -701,13 +711,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
         te += s_priv[w * p.pw + PV + 2 * k + 1];
       }
       if (we == 0) continue;
-      atomicAdd(table + p.off.val + 2ull * site, (unsigned long long)we);
-      atomicAdd(table + p.off.val + 2ull * site + 1, (unsigned long long)te);
+      gadd(p.off.val + 2ull * site, (unsigned long long)we);
+      gadd(p.off.val + 2ull * site + 1, (unsigned long long)te);
       for (uint32_t d = 0; d < nd; ++d) {
         const uint4 st = s_vstate[vd0 + d];
-        if (st.x != FULL) atomicAnd(table + p.off.ones + 4ull * site + d, (unsigned long long)st.x);
-        if (st.y != FULL) atomicAnd(table + p.off.zeros + 4ull * site + d, (unsigned long long)st.y);
-        if (st.z != 1u) atomicAnd(table + p.off.scalar + 4ull * site + d, 0ull);
+        if (st.x != FULL) gand(p.off.ones + 4ull * site + d, (unsigned long long)st.x);
+        if (st.y != FULL) gand(p.off.zeros + 4ull * site + d, (unsigned long long)st.y);
+        if (st.z != 1u) gand(p.off.scalar + 4ull * site + d, 0ull);
       }
     }
   }

@@ -63,6 +63,9 @@ SIGNATURES = {
     "sassi_nccl_comm_destroy": (_i, [_vp]),
     "sassi_kernel_launches": (_i, [_vp, ctypes.POINTER(_u64)]),
     "sassi_enable_dynamic_pcs": (_i, [_vp, _u32]),
+    "sassi_ipc_table_handle": (_i, [_vp, _vp]),
+    "sassi_add_peer_table": (_i, [_vp, _vp]),
+    "sassi_clear_peer_tables": (_i, [_vp]),
     "sassi_read_dynamic_pcs": (_i, [_vp, _vp, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u64), _vp]),
     "sassi_ik_create": (_i, [ctypes.POINTER(_vp), _i, _u32, _u64, _i]),
     "sassi_ik_destroy": (None, [_vp]),
@@ -258,6 +261,21 @@ def sassi_read_dynamic_pcs(ctx: int, stream=None):
     return out[:n.value], dropped.value
 
 
+def sassi_ipc_table_handle(ctx: int) -> bytes:
+    buf = ctypes.create_string_buffer(64)
+    _check(lib().sassi_ipc_table_handle(ctx, buf))
+    return buf.raw
+
+
+def sassi_add_peer_table(ctx: int, handle: bytes) -> None:
+    buf = ctypes.create_string_buffer(bytes(handle), 64)
+    _check(lib().sassi_add_peer_table(ctx, buf))
+
+
+def sassi_clear_peer_tables(ctx: int) -> None:
+    _check(lib().sassi_clear_peer_tables(ctx))
+
+
 def sassi_kernel_launches(ctx: int) -> int:
     n = _u64()
     _check(lib().sassi_kernel_launches(ctx, ctypes.byref(n)))
@@ -326,6 +344,17 @@ class Context:
 
     def read_dynamic_pcs(self, stream=None):
         return sassi_read_dynamic_pcs(self.handle, stream)
+
+    def ipc_table_handle(self) -> bytes:
+        """CUDA IPC handle of this context's table image (for the fused merge)."""
+        return sassi_ipc_table_handle(self.handle)
+
+    def add_peer_table(self, handle: bytes) -> None:
+        """Fold into a peer's table image too (fused fold + merge over peer memory)."""
+        sassi_add_peer_table(self.handle, handle)
+
+    def clear_peer_tables(self) -> None:
+        sassi_clear_peer_tables(self.handle)
 
     def kernel_launches(self) -> int:
         return sassi_kernel_launches(self.handle)
