@@ -212,9 +212,10 @@ uint32_t sm_var_words(uint32_t H) {
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
 }
 
-// kDyn: the insert-on-miss table of unregistered pcs is enabled (a separate instantiation, so the
-// registered-only kernels carry none of its code)
-template <uint32_t H, bool kDyn>
+// kExt: the extended instantiation, used when the insert-on-miss table of unregistered pcs is
+// enabled (p.dyn_cap) and / or the flush also updates peers' images (p.n_peers); the plain kernels
+// carry none of that code
+template <uint32_t H, bool kExt>
 __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
   using Ly = SmLayout<H>;
@@ -243,7 +244,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
   if (H & SASSI_H_MEMDIV)
     for (uint32_t i = tid; i < 1024 * p.npcm; i += blockDim.x) s_pcm[i] = 0;
-  if (kDyn)
+  if (kExt && p.dyn_cap)
     for (uint32_t i = tid; i < kDynLocal; i += blockDim.x) {
       s_dkey[i] = EMPTY_KEY;
       s_dcnt[i] = 0;
@@ -285,11 +286,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   // travel over NVLink to the other GPUs' images, so no collective runs after the fold)
   auto gadd = [&](uint64_t off, unsigned long long v) {
     atomicAdd(table + off, v);
-    for (uint32_t j = 0; j < p.n_peers; ++j) atomicAdd(p.peers[j] + off, v);
+    if (kExt)
+      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAdd(p.peers[j] + off, v);
   };
   auto gand = [&](uint64_t off, unsigned long long v) {
     atomicAnd(table + off, v);
-    for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd(p.peers[j] + off, v);
+    if (kExt)
+      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd(p.peers[j] + off, v);
   };
 
   // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239). Returns the
@@ -306,7 +309,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     known = valid && e.x == h.x && h.x != EMPTY_KEY;
     c_unk += valid && !known;
     c_inv += known && h.z == 0;
-    if (kDyn) {  // dynamic sites: each lane adds its own unregistered record to the CTA's cache
+    if (kExt && p.dyn_cap) {  // dynamic sites: each lane adds its own unregistered record to the CTA's cache
       if (valid && !known) {
         bool done = false;
         if (h.x != EMPTY_KEY) {
@@ -644,7 +647,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
 
   // ---- flush: sum the warps' private counters, fold into the global u64 image ----
   if (tid < 4 && s_diag[tid]) gadd(tid, (unsigned long long)s_diag[tid]);
-  if (kDyn)
+  if (kExt && p.dyn_cap)
     for (uint32_t i = tid; i < kDynLocal; i += blockDim.x)
       if (s_dkey[i] != EMPTY_KEY && s_dcnt[i])
         dyn_insert(s_dkey[i], s_dcnt[i], s_dthr[i], p.dyn_keys, p.dyn_vals, p.dyn_cap, p.dyn_lg);
@@ -732,9 +735,9 @@ __global__ void dyn_reset_kernel(uint32_t* keys, unsigned long long* vals, uint3
 
 using KernelFn = void (*)(const ConsumeParams);
 
-template <uint32_t H, bool kDyn>
+template <uint32_t H, bool kExt>
 KernelFn kernel_for() {
-  return consume_kernel<H, kDyn>;
+  return consume_kernel<H, kExt>;
 }
 
 template <uint32_t... Hs>
@@ -744,7 +747,7 @@ KernelFn pick(uint32_t mask, bool dyn, std::integer_sequence<uint32_t, Hs...>) {
   return fn;
 }
 
-// one instantiation per non-empty handler set (1..31), with and without the dynamic-pc table
+// one instantiation per non-empty handler set (1..31), plain and extended (dynamic pcs / peers)
 KernelFn select_kernel(uint32_t mask, bool dyn) {
   if (mask == 0 || mask > SASSI_H_EVERY) return nullptr;
   return pick(mask, dyn, std::make_integer_sequence<uint32_t, SASSI_H_EVERY>{});
@@ -773,7 +776,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
 }
 
 int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
-  KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0);
+  KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0 || p.n_peers != 0);
   if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
   if ((void*)fn != c->launch_fn || c->smem_bytes != c->launch_smem) {  // configure once per kernel
     {
