@@ -388,8 +388,9 @@ def main():
 
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
-    if not args.no_e2e and rank == 0 and world == 1:
-        e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev)
+    if not args.no_e2e:  # every rank at once on its own shard; the merge is inside the step at N > 1
+        e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev, comm=comm, world=world,
+                          launched=launched)
 
     cpu = None
     if not args.no_cpu_baseline and rank == 0 and world == 1:
@@ -563,10 +564,13 @@ def measure_online_trace(dev, slow=None):
     return out
 
 
-def measure_e2e(rec, P, mask, n_e2e, dev):
+def measure_e2e(rec, P, mask, n_e2e, dev, comm=None, world=1, launched=False):
     """records/s through sassi_consume_host: pinned host buffers of the first n_e2e records, the
-    H2D copies (double-buffered inside the library) and the table read-back inside the timing."""
+    H2D copies (double-buffered inside the library) and the table read-back inside the timing.
+    At N > 1 every rank does the same on its own shard at the same time (after a barrier), the
+    step includes the NCCL merge, and the time is the maximum over ranks."""
     import torch
+    import torch.distributed as dist
     from paper_conf_isca_stephensonhlejn15_b200 import sassi
     n_e2e = (n_e2e // 256) * 256
     cb = rec["chunk_base"][: n_e2e // 256 + 1]
@@ -578,25 +582,47 @@ def measure_e2e(rec, P, mask, n_e2e, dev):
     ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=dev.index)
     stream = torch.cuda.current_stream(dev)
     out = np.zeros(ctx.layout["total"], np.uint64)
-    for _ in range(2):
+    cm = None
+    if comm is not None:  # a communicator of its own for this context
+        uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if not launched or dist.get_rank() == 0:
+            uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
+        if launched:
+            dist.broadcast(uid, 0)
+        cm = sassi.sassi_nccl_comm_create(world, dist.get_rank() if launched else 0,
+                                          bytes(uid.cpu().numpy()), dev.index)
+
+    def one():
         ctx.reset(stream)
         ctx.consume_host(h, stream=stream)
+        if cm is not None:
+            ctx.merge(cm, stream)
         sassi.sassi_read_tables(ctx.handle, out.size, stream, out)
+
+    for _ in range(2):
+        one()
     reps = 3
     torch.cuda.synchronize()
+    if launched:
+        dist.barrier()
     t0 = time.perf_counter()
     for _ in range(reps):
-        ctx.reset(stream)
-        ctx.consume_host(h, stream=stream)
-        sassi.sassi_read_tables(ctx.handle, out.size, stream, out)
+        one()
     el = time.perf_counter() - t0
+    if launched:
+        t = torch.tensor([el], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        el = float(t.item())
+    if cm is not None:
+        sassi.sassi_nccl_comm_destroy(cm)
     ctx.close()
     h2d = 16 * n_e2e + 256 * na + 128 * nv + 16 * (n_e2e // 256 + 1)
-    return {"value": reps * n_e2e / el, "unit": "records/s", "h2d_bytes_per_step": h2d,
-            "d2h_bytes_per_step": 8 * ctx.layout["total"], "records_per_step": n_e2e,
-            "h2d_gbs": reps * h2d / el / 1e9,
-            "note": "pinned host buffers, first %d records; wall clock around consume_host + "
-                    "read_tables (which synchronise)" % n_e2e}
+    return {"value": world * reps * n_e2e / el, "unit": "records/s", "h2d_bytes_per_step": world * h2d,
+            "d2h_bytes_per_step": world * 8 * ctx.layout["total"], "records_per_step": world * n_e2e,
+            "h2d_gbs": world * reps * h2d / el / 1e9,
+            "note": "pinned host buffers, first %d records of each rank's shard; wall clock around "
+                    "consume_host%s + read_tables (which synchronise), max over ranks" % (
+                        n_e2e, " + merge" if cm is not None else "")}
 
 
 if __name__ == "__main__":
