@@ -515,6 +515,9 @@ def measure_slowdown(dev):
         out[name] = r
         ctx.close()
         ik.close()
+    # harmonic mean over the kernels per handler set (the statistic of the paper's Table 3)
+    keys = [k for k in next(iter(out.values())) if k != "base_ms"]
+    out["hmean"] = {k: len(out) / sum(1.0 / out[n][k] for n in out) for k in keys}
     return out
 
 
