@@ -179,3 +179,23 @@ def test_c4_prefix_half_the_sites_unregistered(mask):
     odyn, odrop = oracle.dynamic_pcs(s2, hdr)
     assert dyn == odyn.tolist() and dropped == odrop == 0
     assert len(dyn) == len(s_all) - len(s2)
+
+
+def test_host_buffers_with_dynamic_pcs():
+    """sassi_consume_host (pinned host buffers, staged copies) takes the same extended kernel:
+    tables and dynamic table equal the oracle's."""
+    s, W, hdr, addr, val = random_trace(91, n=20000)
+    rowless = np.array([not (s[i]["flags"] & oracle.F_MEM) and s[i]["n_gpr_dst"] == 0
+                        for i in range(len(s))])
+    s2 = s[~np.isin(s["pc"], s["pc"][rowless][:3])]
+    d = to_device(s2, hdr, addr, val)
+    h = {k: (v.cpu().pin_memory() if hasattr(v, "cpu") else v) for k, v in d.items()}
+    ctx = sassi.Context(s2, W, sassi.SASSI_H_EVERY)
+    ctx.enable_dynamic_pcs(64)
+    ctx.consume_host(h)
+    t = ctx.read_tables()
+    dyn, dropped = ctx.read_dynamic_pcs()
+    ctx.close()
+    assert diff_tables(t, oracle.run(s2, W, sassi.SASSI_H_EVERY, hdr, addr, val), len(s2), W) is None
+    odyn, odrop = oracle.dynamic_pcs(s2, hdr)
+    assert as_list(dyn) == odyn.tolist() and dropped == odrop
