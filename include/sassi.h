@@ -294,7 +294,8 @@ int sassi_merge(struct sassi_ctx* ctx, void* nccl_comm, void* stream);
  * stream synchronise), then sassi_read_tables anywhere. The dynamic-pc table and the inline
  * handlers of sassi_ik_run are not included (use sassi_merge for those).
  * sassi_add_peer_table: only before the first consume or right after sassi_reset; the peer's image
- * must have this context's layout (EMISMATCH otherwise); at most 7 peers (ENOSPC).
+ * must have this context's layout (EMISMATCH otherwise); at most 7 peers (ENOSPC). While peers are
+ * attached the handler set cannot change (sassi_attach_handler: ESTATE).
  * sassi_clear_peer_tables synchronises the device and closes the handles. */
 #define SASSI_IPC_HANDLE_BYTES 64
 int sassi_ipc_table_handle(struct sassi_ctx* ctx, void* handle_out);
