@@ -22,6 +22,10 @@
 
 #include "common.cuh"
 
+#ifndef SASSI_HDR_DEPTH
+#define SASSI_HDR_DEPTH 3  // header batches in flight per warp (header-only handler sets)
+#endif
+
 namespace sassi {
 namespace {
 
@@ -404,7 +408,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     // ---- header-only handler sets: each warp takes one contiguous range of records (so its
     // per-thread-count accumulator stays on one trace warp for thousands of records) and walks it
     // in 32-record batches, headers loaded kDepth batches ahead ----
-    constexpr uint32_t kDepth = 3;
+    constexpr uint32_t kDepth = SASSI_HDR_DEPTH;
     const uint32_t per = (p.n + 32u * nw - 1u) / (32u * nw) * 32u;  // records per warp
     const uint32_t R0 = min((blockIdx.x * kWarpsPerCta + wib) * per, p.n), R1 = min(R0 + per, p.n);
     if (lane == 0) c_rec += R1 - R0;
@@ -417,7 +421,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     for (uint32_t k = 0; k < kDepth; ++k) q[k] = hload(first_rec(k));
     uint32_t it = 0;  // iterations since the vertical counters were last folded
     for (uint32_t t = 0;; t += kDepth) {
-      if ((H & SASSI_H_INSTCOUNT) && kVertical && ++it == 6) {  // <= 15 additions between folds
+      // fold every floor(15 / kDepth) iterations: <= 15 additions between folds
+      if ((H & SASSI_H_INSTCOUNT) && kVertical && ++it == 15 / kDepth + 1) {
         flush_planes();
         it = 1;
       }
