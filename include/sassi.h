@@ -194,14 +194,15 @@ int sassi_ctx_create(struct sassi_ctx** out, int device, const sassi_site* sites
 void sassi_ctx_destroy(struct sassi_ctx* ctx);
 
 /* Select which handlers run (non-empty subset of SASSI_H_EVERY) — the paper's "what"
- * (L181-L187). Allowed only
- * before the first consume or right after sassi_reset. Errors: EINVAL, ESTATE, ENOSPC. */
+ * (L181-L187). Allowed only before the first consume or right after sassi_reset, and not to a
+ * different set while peer tables are attached. Errors: EINVAL, ESTATE, ENOSPC. */
 int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
 
 /* Keep a per-PC memory-divergence matrix (pcmat, the Fig.6 32x32 matrix of that pc's own records)
  * for k <= SASSI_MAX_PC_MATRICES registered GLOBAL memory sites given by pc (HOST array; k = 0
  * clears the selection). Like sassi_attach_handler: only before the first consume or right after
- * sassi_reset; the selection is part of the site-table checksum sassi_merge compares. Takes
+ * sassi_reset, not while peer tables are attached; the selection is part of the site-table
+ * checksum sassi_merge compares (and of the layout sassi_add_peer_table checks). Takes
  * effect with SASSI_H_MEMDIV attached; costs 4 KB of shared memory per selected pc per CTA.
  * Errors: EINVAL (unknown pc, not a GLOBAL memory site, k too large), ESTATE, ENOSPC. */
 int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
@@ -232,8 +233,9 @@ typedef struct sassi_dyn_pc {
 int sassi_read_dynamic_pcs(struct sassi_ctx* ctx, sassi_dyn_pc* host_out, uint32_t cap_out,
                            uint32_t* n_out, uint64_t* n_dropped, void* stream);
 
-/* Fold n records (DEVICE buffers) into the context's tables; asynchronous, stream-ordered.
- * Tables accumulate across calls until sassi_reset. One kernel launch per 2^29 records (the
+/* Fold n records (DEVICE buffers) into the context's tables (and, with peer tables attached,
+ * into theirs); asynchronous, stream-ordered. Tables accumulate across calls until sassi_reset.
+ * One kernel launch per 2^29 records (the
  * environment variable SASSI_MAX_LAUNCH_RECORDS, read at sassi_ctx_create, lowers that to a
  * multiple of SASSI_CHUNK for tests). Errors: EINVAL, ESTATE (no handler), ECUDA. */
 int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, void* stream);
@@ -249,7 +251,9 @@ int sassi_consume_host(struct sassi_ctx* ctx, const sassi_records* host_recs, ui
 int sassi_index_records(struct sassi_ctx* ctx, const sassi_hdr* hdr, uint64_t n,
                         sassi_chunk_base* chunk_base_out, void* stream);
 
-/* Re-initialise all tables (CUPTI kernel-launch callback analogue, L217). Asynchronous. */
+/* Re-initialise all tables, and the dynamic-pc table when enabled (CUPTI kernel-launch callback
+ * analogue, L217). Asynchronous. With peer tables attached it resets this context's image only:
+ * every rank resets its own, then a barrier, before any rank folds (see sassi_add_peer_table). */
 int sassi_reset(struct sassi_ctx* ctx, void* stream);
 
 /* Copy the table image (sassi_table_layout(...).total words) to HOST memory; synchronises
