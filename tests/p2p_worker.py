@@ -33,6 +33,15 @@ def run_case(name, sites, W, mask, d, want, rank, world):
     for j in range(world):
         if j != rank:
             ctx.add_peer_table(handles[j])
+    # while peers fold into this image its layout is fixed: another handler set or pc selection
+    # is refused
+    for bad in (lambda: sassi.sassi_attach_handler(ctx.handle, sassi.SASSI_H_BRANCH),
+                lambda: ctx.select_memdiv_pcs([])):
+        try:
+            bad()
+            raise AssertionError("layout change accepted with peer tables attached")
+        except sassi.SassiError as e:
+            assert e.status == sassi.SASSI_ESTATE
     for rep in range(2):  # twice: reset between rounds works with peers attached
         ctx.reset()
         torch.cuda.synchronize()
