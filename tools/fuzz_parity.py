@@ -37,8 +37,11 @@ for case in range(n_cases):
         ctx.select_memdiv_pcs([int(s[i]["pc"]) for i in sel])
     if dyn:
         ctx.enable_dynamic_pcs(64)
-    # consume in one piece or in two chunk-aligned pieces
-    if n > 512 and rng.integers(0, 2):
+    # consume in one piece, in two chunk-aligned pieces, or from pinned host buffers
+    how = int(rng.integers(0, 3))
+    if how == 2:
+        ctx.consume_host({k: (v.cpu().pin_memory() if hasattr(v, "cpu") else v) for k, v in d.items()})
+    elif n > 512 and how == 1:
         half = (n // 2) // 256 * 256
         ctx.consume(dict(d, hdr=d["hdr"][:half], chunk_base=d["chunk_base"][: half // 256 + 1], n=half))
         ctx.consume(dict(d, hdr=d["hdr"][half:], chunk_base=d["chunk_base"][half // 256:], n=n - half))
@@ -53,6 +56,12 @@ for case in range(n_cases):
         got = [[int(e["pc"]), int(e["warp_execs"]), int(e["thread_execs"])] for e in dynt]
         if got != odyn.tolist() or dropped != odrop:
             msg = "dynamic table differs"
+    if msg is None and (mask & 8):  # injection-site draws over the per-thread counts (L629)
+        sec = oracle.sections(o, len(s), W)
+        if int(sec["counts"].sum()) > 0:
+            k, sd = int(rng.integers(1, 300)), int(rng.integers(0, 2**62))
+            if not np.array_equal(ctx.sample(k, sd), oracle.sample(sec["counts"], k, sd)):
+                msg = "sampling differs"
     ctx.close()
     if msg is not None:
         fails += 1
