@@ -38,7 +38,7 @@ if PART in ("all", "base"):
     for name, size in (("vecadd", 12800), ("bfs", 4096), ("sgemm", 32), ("stencil", 64)):
         ik = sassi.InstrumentedKernel(name, size)
         ctx = ik.context(sassi.SASSI_H_EVERY)
-        for mode in (0, 1, 2, 4, 8, 16, 15, 31, sassi.SASSI_IK_NULL_ABI):
+        for mode in (0, 1, 2, 4, 8, 16, 15, 31, sassi.SASSI_IK_NULL_ABI, 1024 | 1, 1024 | 2, 1024 | 15, 1024 | 31):
             ctx.reset()
             ik.run(mode, ctx if mode & 31 else None)
         ik.trace(ctx)
