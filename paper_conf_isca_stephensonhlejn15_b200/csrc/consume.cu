@@ -25,6 +25,12 @@
 #ifndef SASSI_HDR_DEPTH
 #define SASSI_HDR_DEPTH 3  // header batches in flight per warp (header-only handler sets)
 #endif
+#ifndef SASSI_HASH_LG
+#define SASSI_HASH_LG 11     // memdiv distinctness check: 2^11 bit buckets per warp (256 B)
+#endif
+#ifndef SASSI_HASH_ROUNDS
+#define SASSI_HASH_ROUNDS 2  // hash rounds (different multipliers) before the exact sort
+#endif
 
 namespace sassi {
 namespace {
@@ -106,18 +112,36 @@ __device__ __forceinline__ void count_sorted(T v, uint32_t n, uint32_t lane, uin
   *out_l = __popc(__ballot_sync(FULL, new_l));
 }
 
+// One round of the distinctness check of a gather row: every lane of G sets bit h(line) of the
+// warp's 2^SASSI_HASH_LG-bit shared-memory bitmap with an atomic OR that returns the old word. If
+// no lane finds its bit already set, the lines of G hash to pairwise different buckets, so they
+// are pairwise distinct (equal lines hash alike). The lanes then clear their words again.
+__device__ __forceinline__ bool lines_distinct(uint32_t line, bool in, uint32_t* bm, uint32_t mul) {
+  const uint32_t h = (line * mul) >> (32 - SASSI_HASH_LG);
+  uint32_t* const w = bm + (h >> 5);
+  const uint32_t bit = 1u << (h & 31u);
+  const uint32_t old = in ? atomicOr(w, bit) : 0u;
+  const bool ok = !__any_sync(FULL, (old & bit) != 0u);
+  __syncwarp();
+  if (in) *w = 0u;
+  __syncwarp();
+  return ok;
+}
+
 // Fig.6 for one warp-wide address row: n = |G|, s = distinct (addr >> 5), L = distinct (addr >> 7)
 // over the lanes of G (the count of Fig.6's leader-election loop, l.16-26).
 //  - window path: every sector of G within the 32-sector (1 KB, 8-line) window that starts at the
 //    line holding the lowest sector (same high word): the window bitmap is OR-reduced across the
 //    warp (REDUX), s = its popcount, L = the popcount of its nibbles OR-folded (a nibble = a line).
-//  - otherwise, when all high words agree: sort the 32-bit keys across the warp (bitonic) with the
+//  - otherwise, when all high words agree (gathers): if a hashed bitmap shows the lines of G to be
+//    pairwise distinct, s = L = |G| (lines_distinct, two rounds); else sort the 32-bit keys across
+//    the warp (bitonic) with the
 //    lanes outside G padded to the maximum so they sort last, and count positions < n whose key
 //    differs from the previous one; lines come from the same sorted sectors (>> 2 keeps order).
 //  - rows whose sectors differ in the high word return false and go to memdiv_row64 (64-bit keys),
 //    called once per such row outside the unrolled row loop to keep that loop's code small.
-__device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t lane, uint32_t* out_s,
-                                             uint32_t* out_l) {
+__device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t lane, uint32_t* bm,
+                                             uint32_t* out_s, uint32_t* out_l) {
   const bool in = (G >> lane) & 1u;
   const uint64_t sec = a >> 5;
   const uint32_t slo = (uint32_t)sec, shi = (uint32_t)(sec >> 32);
@@ -132,6 +156,16 @@ __device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t la
     return true;
   }
   if (!__all_sync(FULL, same_hi)) return false;
+  // scattered rows (gathers): if the lines of G are pairwise distinct, so are the sectors, and
+  // s = L = |G| with no sort; a hash collision or a repeated line falls through to the sort
+  if (SASSI_HASH_ROUNDS >= 1 && lines_distinct(slo >> 2, in, bm, 0x9E3779B1u)) {
+    *out_s = *out_l = __popc(G);
+    return true;
+  }
+  if (SASSI_HASH_ROUNDS >= 2 && lines_distinct(slo >> 2, in, bm, 0x85EBCA6Bu)) {
+    *out_s = *out_l = __popc(G);
+    return true;
+  }
   count_sorted(warp_sort<uint32_t>(in ? slo : FULL, lane), __popc(G), lane, out_s, out_l);
   return true;
 }
@@ -202,7 +236,9 @@ struct SmLayout {
   static constexpr uint32_t kImix = 8;                                  // 8 u64 (instmix totals)
   static constexpr uint32_t kH32 = 24;                                  // [32][32] u32 (memdiv)
   static constexpr uint32_t kH128 = kH32 + 1024;                        // [32][32] u32 (memdiv)
-  static constexpr uint32_t kBar = kMem ? kH128 + 1024 : 24;            // [warps] u64 (value)
+  static constexpr uint32_t kHbm = kH128 + 1024;  // [warps][2^LG / 32] distinctness bitmaps
+  static constexpr uint32_t kHbmWords = SASSI_HASH_ROUNDS ? (1u << SASSI_HASH_LG) / 32 : 0u;
+  static constexpr uint32_t kBar = kMem ? kHbm + kWarpsPerCta * kHbmWords : 24;
   static constexpr uint32_t kVbuf = kVal ? ((kBar + 2 * kWarpsPerCta + 31) & ~31u) : kBar;
   static constexpr uint32_t kVar = kVbuf + (kVal ? kWarpsPerCta * kVbufWords : 0u);  // hash, ...
   static_assert(kVbuf % 32 == 0 || !kVal, "value buffers must be 128 B aligned");
@@ -211,7 +247,8 @@ struct SmLayout {
 // host mirror of SmLayout<H>::kVar
 uint32_t sm_var_words(uint32_t H) {
   const bool mem = H & SASSI_H_MEMDIV, val = H & SASSI_H_VALUE;
-  const uint32_t bar = mem ? 24 + 2048 : 24;
+  const uint32_t hbm = SASSI_HASH_ROUNDS ? (1u << SASSI_HASH_LG) / 32 : 0u;
+  const uint32_t bar = mem ? 24 + 2048 + kWarpsPerCta * hbm : 24;
   const uint32_t vbuf = val ? ((bar + 2 * kWarpsPerCta + 31) & ~31u) : bar;
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
 }
@@ -263,6 +300,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   uint32_t* const wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
   uint4* const vbuf = reinterpret_cast<uint4*>(sm + kSmVbuf + wib * kVbufWords);
   uint64_t* const vbar = reinterpret_cast<uint64_t*>(sm + kSmBar) + wib;
+  uint32_t* const hbm = sm + Ly::kHbm + wib * Ly::kHbmWords;  // this warp's distinctness bitmap
   uint32_t vphase = 0;
   const uint32_t PB = 4 * p.nb, PV = 4 * p.nb + 4 * p.nm;
   const uint32_t n_units = (p.n + SASSI_CHUNK - 1) / SASSI_CHUNK;
@@ -532,7 +570,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
             for (int k = 0; k < 4; ++k) {
               if (g[k]) {
                 uint32_t s, L;
-                if (memdiv_row32(a[k], g[k], lane, &s, &L)) {
+                if (memdiv_row32(a[k], g[k], lane, hbm, &s, &L)) {
                   if (lane == jj[k]) {
                     my_s = s;
                     my_l = L;
@@ -753,10 +791,17 @@ KernelFn pick(uint32_t mask, bool dyn, std::integer_sequence<uint32_t, Hs...>) {
 }
 
 // one instantiation per non-empty handler set (1..31), plain and extended (dynamic pcs / peers)
+#ifndef SASSI_ONLY_H
 KernelFn select_kernel(uint32_t mask, bool dyn) {
   if (mask == 0 || mask > SASSI_H_EVERY) return nullptr;
   return pick(mask, dyn, std::make_integer_sequence<uint32_t, SASSI_H_EVERY>{});
 }
+#else  // development builds (SASS inspection): one handler set only
+KernelFn select_kernel(uint32_t mask, bool dyn) {
+  if (mask != SASSI_ONLY_H) return nullptr;
+  return dyn ? kernel_for<SASSI_ONLY_H, true>() : kernel_for<SASSI_ONLY_H, false>();
+}
+#endif
 
 }  // namespace
 
