@@ -1,17 +1,24 @@
 #!/usr/bin/env python3
 """bench.py — records/s and HBM GB/s of the SASSI handler fold on B200 (BASELINE.json metric).
 
-Workload (N=1): config c3 of BASELINE.json (the largest configuration that fits one GPU; c5, the
-8-GPU configuration, does not): an SGEMM/stencil-shaped trace of 10^8 warp-instruction records
-(~19 GB in HBM, >> the 126 MB L2, so no flush is needed between steps), all four handlers
-attached. One step = the whole hot path: sassi_reset (CUPTI launch-callback analogue) +
-sassi_consume (fused fold) + sassi_sample_sites (1,000 injection sites, L629) [+ sassi_merge over
-NCCL when N > 1]. Weak scaling: each rank folds its own 10^8-record shard (its own warp ids).
+N = 1 (default): config c3 of BASELINE.json (the largest configuration that fits one GPU): an
+SGEMM/stencil-shaped trace of 10^8 warp-instruction records (~19 GB in HBM, >> the 126 MB L2, so
+no flush is needed between steps), all four handlers attached. One step = the whole hot path:
+sassi_reset (CUPTI launch-callback analogue) + sassi_consume (fused fold) + sassi_sample_sites
+(1,000 injection sites, L629).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--workload c3|c2|c4]
+N > 1: config c5, the configuration the metric quotes for 8 GPUs: ~4x10^9 records in 8 warp shards,
+strong scaling (the total is fixed; rank r folds shards r, r+N, ...), the per-rank tables merged
+by sassi_merge (one NCCL allreduce) before the 1,000 draws. The line carries c5's 1-GPU time T_1
+(rank 0 alone folds all 8 shards afterwards, same protocol) so E_N = T_1 / (N T_N) can be formed,
+and a weak-scaling secondary (every rank folds its own c3-shaped 10^8-record shard + the merge).
 
---impl reference times the oracle (plain single-threaded C++, oracle/) on the host cores on a
-bounded sample of the same workload — the only reference implementation this tier has.
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--workload c2|c3|c4|c5]
+
+--gpus N without torchrun re-launches this script under torch.distributed.run with N ranks (one
+per GPU, rendezvous on 127.0.0.1). --impl reference times the oracle (plain single-threaded C++,
+oracle/) on the host cores on a bounded sample of the same workload — the only reference
+implementation this tier has.
 """
 from __future__ import annotations
 
@@ -39,7 +46,10 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="c3", choices=["c2", "c3", "c4", "c5"])
+    ap.add_argument("--workload", default=None, choices=["c2", "c3", "c4", "c5"],
+                    help="default: c3 at N = 1, c5 at N > 1")
+    ap.add_argument("--selftest-dist", action="store_true",
+                    help="launch / rendezvous / max-over-ranks plumbing only (gloo without a GPU)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-slowdown", action="store_true")
@@ -52,6 +62,78 @@ def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return rank, world, local
+
+
+def self_launch(n):
+    """`--gpus N` outside torchrun: run this script under torch.distributed.run with N ranks on this
+    node (rendezvous on 127.0.0.1, a free port); returns its exit code. Rank 0 prints the line."""
+    import socket
+    import subprocess
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=%d" % n,
+           "--master-addr=127.0.0.1", "--master-port=%d" % port, os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def max_over_ranks(x, dev=None):
+    """Maximum of a float over all ranks (device timing rule: the job time is the slowest rank's)."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()):
+        return x
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def sum_over_ranks(x, dev=None):
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()):
+        return x
+    t = torch.tensor([int(x)], dtype=torch.int64, device=dev)
+    dist.all_reduce(t)
+    return int(t.item())
+
+
+def host_info():
+    """nproc and the CPU model of the box the oracle baseline runs on."""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+def run_selftest_dist(args, rank, world):
+    """The multi-rank plumbing of this script without a GPU: process group (nccl with CUDA, else
+    gloo), barrier, a per-rank timing reduced as the maximum over ranks, one line from rank 0."""
+    import torch
+    import torch.distributed as dist
+    backend = "nccl" if torch.cuda.is_available() else "gloo"
+    dev = None
+    if backend == "nccl":
+        torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", "0")))
+        dev = torch.device("cuda", torch.cuda.current_device())
+    if world > 1:
+        dist.init_process_group(backend)
+        dist.barrier()
+    t0 = time.perf_counter()
+    time.sleep(0.01 * (rank + 1))
+    el = max_over_ranks(time.perf_counter() - t0, dev)
+    ranks = sum_over_ranks(1, dev)
+    if rank == 0:
+        print(json.dumps({"selftest": "dist", "n_gpus": world, "ranks_reporting": ranks,
+                          "backend": backend if world > 1 else "none", "max_over_ranks_s": el}),
+              flush=True)
+    if world > 1:
+        dist.destroy_process_group()
 
 
 def measured_peaks():
@@ -146,14 +228,15 @@ def algorithmic_bytes(rec, handlers):
     return b, n_glob
 
 
-def run_reference(args, rank, world):
-    """Oracle on the host cores, on a bounded sample of the same workload (rank 0 only)."""
+def run_reference(args, rank, world, workload):
+    """Oracle on the host cores, on a bounded sample of the same workload (rank 0 only; under
+    torchrun the other ranks exit without work)."""
     if rank != 0:
         return
     import oracle
     from paper_conf_isca_stephensonhlejn15_b200 import gen
-    P, limit, desc = workload_program(args.workload, 1)
-    mask = gen.PRESETS[args.workload][2]
+    P, limit, desc = workload_program(workload, 1)
+    mask = gen.PRESETS[workload][2]
     sample_n = 1 << 21
     rec = gen.generate_host(P, sample_n, 0, 1024)
     times = []
@@ -166,12 +249,14 @@ def run_reference(args, rank, world):
     v = args.steps * rec["n"] / tmax
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "records/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * tmax / args.steps, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": {"workload": args.workload + ": " + desc, "sample_records": rec["n"]},
-            "cpu_baseline": {"value": v, "unit": "records/s", "cores": 1, "kind": "oracle",
-                             "sample": "first %d records (warps 0..1023) of %s per step" %
-                                       (rec["n"], args.workload)},
+            "ms_per_step": 1e3 * tmax / args.steps, "higher_is_better": True,
+            "scaling": "weak" if world == 1 else "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": workload + ": " + desc, "sample_records": rec["n"]},
+            "cpu_baseline": dict({"value": v, "unit": "records/s", "cores": 1, "threads": 1,
+                                  "kind": "oracle",
+                                  "sample": "first %d records (warps 0..1023) of %s per step" %
+                                            (rec["n"], workload)}, **host_info()),
             "e2e": {"value": v, "unit": "records/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -196,82 +281,119 @@ def cpu_baseline(args, d_rec, mask, P):
         el = time.perf_counter() - t0
         if el > 10.0 or reps >= 30:
             break
-    return {"value": reps * n / el, "unit": "records/s", "cores": 1, "kind": "oracle",
-            "sample": "first %d records of the %s stream, %d repetition(s), %.1f s" %
-                      (n, args.workload, reps, el)}
+    return dict({"value": reps * n / el, "unit": "records/s", "cores": 1, "threads": 1,
+                 "kind": "oracle",
+                 "sample": "first %d records of the %s stream, %d repetition(s), %.1f s" %
+                           (n, args.workload, reps, el)}, **host_info())
+
+
+def nccl_comm(world, rank, local, dev):
+    """A communicator of libsassi's own (its NCCL), the unique id broadcast over torch.distributed."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+    if rank == 0:
+        uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
+    if dist.is_initialized():
+        dist.broadcast(uid, 0)
+    return sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
+
+
+def fold_c5_shards(args, shards, P, mask, dev, local, job=None):
+    """Fold c5 warp shards one by one into `job` (a Context, created if None): each shard is
+    generated in HBM (untimed), warmed up, timed over --steps passes of reset + consume on a scratch
+    context (CUDA events on the launching stream), then folded once more into the job.
+    -> (job, per-shard mean consume ms, records, algorithmic bytes)."""
+    import torch
+    from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
+    stream = torch.cuda.current_stream(dev)
+    scratch = None
+    consume_ms, n_total, alg_total = [], 0, 0
+    for shard in shards:
+        rec = gen.generate_device(P, None, shard * 16384, 16384, device=dev)
+        if job is None:
+            job = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
+        if scratch is None:
+            scratch = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
+        b, _ = algorithmic_bytes(rec, mask)
+        for _ in range(args.warmup):
+            scratch.reset(stream)
+            scratch.consume(rec, stream=stream)
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)]
+        for a, e in evs:
+            scratch.reset(stream)
+            a.record(stream)
+            scratch.consume(rec, stream=stream)
+            e.record(stream)
+        job.consume(rec, stream=stream)
+        torch.cuda.synchronize(dev)
+        consume_ms.append(statistics.mean(a.elapsed_time(e) for a, e in evs))
+        n_total += rec["n"]
+        alg_total += b
+        del rec
+        torch.cuda.empty_cache()
+    scratch.close()
+    return job, consume_ms, n_total, alg_total
 
 
 def run_c5(args, rank, world, local):
     """Config c5 as the metric quotes it: ~4x10^9 records in 8 warp shards of 16,384 warps. Rank r
-    folds shards r, r+N, ... (strong scaling: the total is fixed); each shard is generated in HBM
-    (untimed), its fold is timed over --steps passes (reset + consume, CUDA events), and one more
-    pass accumulates into the job's context; the job time is the sum over shards plus the final
-    1,000-site sampling (+ the NCCL merge when N > 1), max over ranks."""
+    folds shards r, r+N, ... (strong scaling: the total is fixed); the job time is the sum over the
+    rank's shards of the timed fold + the NCCL merge (N > 1) + the final 1,000-site sampling, max
+    over ranks. At N > 1 rank 0 then folds all 8 shards alone (same protocol: T_1) and every rank
+    runs the c3 weak-scaling measurement (secondary key)."""
     import torch
     import torch.distributed as dist
-    from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
-    torch.cuda.set_device(local)
+    from paper_conf_isca_stephensonhlejn15_b200 import gen
     dev = torch.device("cuda", local)
-    launched = "RANK" in os.environ
-    if launched:
-        dist.init_process_group("nccl", device_id=dev)
     P, limit, mask, desc = gen.preset("c5")
     stream = torch.cuda.current_stream(dev)
-    job = None
-    scratch = None
-    t_shards = 0.0
-    n_total = 0
-    alg_total = 0
-    consume_ms = []
+    comm = nccl_comm(world, rank, local, dev) if world > 1 else None
+    draws = torch.empty(N_DRAWS * 32, dtype=torch.uint8, device=dev)
+    status = torch.zeros(1, dtype=torch.int32, device=dev)
     with ClockSampler(local) as clk:
-        for shard in range(rank, 8, world):
-            rec = gen.generate_device(P, None, shard * 16384, 16384, device=dev)
-            if job is None:
-                job = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
-                scratch = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
-            b, _ = algorithmic_bytes(rec, mask)
-            for _ in range(args.warmup):
-                scratch.reset(stream)
-                scratch.consume(rec, stream=stream)
-            evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                   for _ in range(args.steps)]
-            for a, e in evs:
-                scratch.reset(stream)
-                a.record(stream)
-                scratch.consume(rec, stream=stream)
-                e.record(stream)
-            job.consume(rec, stream=stream)
-            torch.cuda.synchronize()
-            ms = statistics.mean(a.elapsed_time(e) for a, e in evs)
-            consume_ms.append(ms)
-            t_shards += ms / 1e3
-            n_total += rec["n"]
-            alg_total += b
-            del rec
-            torch.cuda.empty_cache()
+        job, consume_ms, n_total, alg_total = fold_c5_shards(args, range(rank, 8, world), P, mask,
+                                                             dev, local)
+        if world > 1:
+            dist.barrier()
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t0.record(stream)
-        if world > 1:
-            uid = torch.zeros(128, dtype=torch.uint8, device=dev)
-            if rank == 0:
-                uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
-            dist.broadcast(uid, 0)
-            comm = sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
+        if comm is not None:
             job.merge(comm, stream)
-        job.sample(N_DRAWS, 20150617, stream)
+        job.sample_device(draws, status, N_DRAWS, 20150617, stream)
         t1.record(stream)
-        torch.cuda.synchronize()
-    t_job = t_shards + t0.elapsed_time(t1) / 1e3
-    if launched:
-        tt = torch.tensor([t_job], device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        t_job = float(tt.item())
-        nt = torch.tensor([n_total], device=dev, dtype=torch.int64)
-        dist.all_reduce(nt)
-        n_total = int(nt.item())
-        at = torch.tensor([alg_total], device=dev, dtype=torch.int64)
-        dist.all_reduce(at)
-        alg_total = int(at.item())
+        torch.cuda.synchronize(dev)
+    assert int(status.item()) == 0, "c5: nothing to sample"
+    t_tail = t0.elapsed_time(t1) / 1e3
+    t_shards = sum(consume_ms) / 1e3
+    t_job = max_over_ranks(t_shards + t_tail, dev)
+    n_total = sum_over_ranks(n_total, dev)
+    alg_total = sum_over_ranks(alg_total, dev)
+    launches = job.kernel_launches()
+    n_sites = len(job.sites)
+    job.close()
+    t1_job = t1_shard_ms = None
+    weak = None
+    if world > 1:
+        dist.barrier()
+        if rank == 0:  # T_1: the same job on one GPU (all 8 shards, no merge)
+            j1, ms1, _, _ = fold_c5_shards(args, range(8), P, mask, dev, local)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            j1.sample_device(draws, status, N_DRAWS, 20150617, stream)
+            b.record(stream)
+            torch.cuda.synchronize(dev)
+            t1_job = sum(ms1) / 1e3 + a.elapsed_time(b) / 1e3
+            t1_shard_ms = ms1
+            j1.close()
+        dist.barrier()
+        weak = run_weak(args, rank, world, local, "c3", extras=False, comm=comm,
+                        steps=min(args.steps, 10))
+    if comm is not None:
+        from paper_conf_isca_stephensonhlejn15_b200 import sassi
+        sassi.sassi_nccl_comm_destroy(comm)
     if rank == 0:
         peak, peak_src = measured_peaks()
         per_gpu_alg = alg_total / world
@@ -281,57 +403,54 @@ def run_c5(args, rank, world, local):
                 "data": "synthetic",
                 "config": {"workload": "c5: " + desc + " (8 warp shards of 16,384 warps, folded "
                            "shard by shard; step = all shards + merge + 1000-site sampling)",
-                           "records": n_total, "sites": len(job.sites), "threads": 32 * P.total_warps,
-                           "handlers": mask, "algorithmic_bytes": alg_total,
+                           "records": n_total, "sites": n_sites,
+                           "threads": 32 * P.total_warps, "handlers": mask,
+                           "algorithmic_bytes": alg_total,
                            "l2": "each shard is ~90 GB >> 126 MB L2; no flush",
-                           "parallelism": "dp%d over warp shards" % world},
+                           "parallelism": "dp%d over warp shards%s" % (
+                               world, ", NCCL allreduce merge" if world > 1 else "")},
                 "hbm_gbs": alg_total / t_job / 1e9,
+                "hbm_frac_of_spec_8tbs": per_gpu_alg / t_job / 1e9 / SPEC_HBM_GBS,
                 "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
                              "achieved": per_gpu_alg / t_shards / 1e9, "peak": peak, "unit": "GB/s",
                              "frac": per_gpu_alg / t_shards / 1e9 / peak, "peak_source": peak_src,
-                             "traffic": None, "consume_ms_per_shard": consume_ms},
-                "gpu_launches": job.kernel_launches(), "clocks": clk.result()}
+                             "traffic": ncu_traffic("c5"), "consume_ms_per_shard": consume_ms},
+                "gpu_launches": launches, "clocks": clk.result()}
+        if world > 1:
+            line["strong_scaling"] = {
+                "t1_ms": 1e3 * t1_job, "tN_ms": 1e3 * t_job, "t1_consume_ms_per_shard": t1_shard_ms,
+                "note": "T_1 = rank 0 alone folding all 8 shards + sampling, same protocol, same run; "
+                        "E_N = T_1 / (N T_N) (north_star target >= 0.85)"}
+        if weak:
+            line["weak_scaling"] = weak
+            if "e2e" in weak:
+                line["e2e"] = dict(weak["e2e"], note=weak["e2e"]["note"] + " (c3-shaped shard per rank: "
+                                   "c5's records never exist in host memory at once)")
         print(json.dumps(line), flush=True)
-    job.close()
-    scratch.close()
-    if launched:
-        dist.destroy_process_group()
 
 
-def main():
-    args = parse()
-    rank, world, local = dist_env()
-    if args.impl == "reference":
-        run_reference(args, rank, world)
-        return
-    if args.workload == "c5":
-        run_c5(args, rank, world, local)
-        return
+def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=None):
+    """`workload` (c2 / c3 / c4), each rank folding its own shard of the preset's size (weak scaling:
+    warp ids offset by rank), + the NCCL merge when N > 1, + 1,000 draws. Returns the JSON line on
+    rank 0 (None elsewhere); extras = e2e, cpu_baseline, slowdown, online trace, injection."""
     import torch
     import torch.distributed as dist
     from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
 
-    torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    launched = "RANK" in os.environ  # under torchrun (any world size)
+    steps = args.steps if steps is None else steps
+    launched = dist.is_initialized()
     merge_on = world > 1 or os.environ.get("SASSI_BENCH_FORCE_MERGE") == "1"
-    if launched:
-        dist.init_process_group("nccl", device_id=dev)
-    P, limit, desc = workload_program(args.workload, world)
-    mask = gen.PRESETS[args.workload][2]
+    P, limit, desc = workload_program(workload, world)
+    mask = gen.PRESETS[workload][2]
     per = P.total_warps // world
     rec = gen.generate_device(P, limit, rank * per, per, device=dev)
     n = rec["n"]
     alg_bytes, n_glob = algorithmic_bytes(rec, mask)
     ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
-    comm = None
-    if merge_on:
-        uid = torch.zeros(128, dtype=torch.uint8, device=dev)
-        if rank == 0:
-            uid.copy_(torch.frombuffer(bytearray(sassi.sassi_nccl_get_unique_id()), dtype=torch.uint8))
-        if launched:
-            dist.broadcast(uid, 0)
-        comm = sassi.sassi_nccl_comm_create(world, rank, bytes(uid.cpu().numpy()), local)
+    own_comm = None
+    if merge_on and comm is None:
+        comm = own_comm = nccl_comm(world, rank, local, dev)
     stream = torch.cuda.current_stream(dev)
     sample = bool(mask & 8)
     # draws stay on the device inside the timed steps (stream-ordered, no host round trip per step)
@@ -358,11 +477,11 @@ def main():
     torch.cuda.synchronize()
     launches0 = ctx.kernel_launches()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-           for _ in range(args.steps)]
+           for _ in range(steps)]
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         t_start.record(stream)
-        for k in range(args.steps):
+        for k in range(steps):
             step(*evs[k])
         t_end.record(stream)
         torch.cuda.synchronize()
@@ -374,14 +493,10 @@ def main():
         assert int(draw_status.item()) == 0, "sampling: no eligible dynamic instruction"
         host_draws = ctx.sample(N_DRAWS, 20150616, stream)
         assert draws.cpu().numpy().tobytes() == host_draws.tobytes(), "device draws differ"
-    ms = t_start.elapsed_time(t_end)
+    ms = max_over_ranks(t_start.elapsed_time(t_end), dev)
     consume_ms = [a.elapsed_time(b) for a, b in evs]
-    if launched:
-        tt = torch.tensor([ms], device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
     sec = ms / 1e3
-    value = world * n * args.steps / sec
+    value = world * n * steps / sec
     consume_avg_s = statistics.mean(consume_ms) / 1e3
     peak, peak_src = measured_peaks()
     achieved = alg_bytes / consume_avg_s / 1e9
@@ -392,62 +507,81 @@ def main():
         e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev, comm=comm, world=world,
                           launched=launched)
 
-    cpu = None
-    if not args.no_cpu_baseline and rank == 0 and world == 1:
+    cpu = slow = online = inj = None
+    if extras and not args.no_cpu_baseline and rank == 0 and world == 1:
         cpu = cpu_baseline(args, rec, mask, P)
-
-    slow = online = None
-    if not args.no_slowdown and rank == 0:
+    if extras and not args.no_slowdown and rank == 0:
         slow = measure_slowdown(dev)
         online = measure_online_trace(dev, slow)
-    inj = None
-    if not args.no_injection and rank == 0:
+    if extras and not args.no_injection and rank == 0:
         inj = measure_injection(dev)
-
-    if rank == 0:
-        line = {
-            "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
-            "data": "synthetic",
-            "config": {"workload": args.workload + ": " + desc + ", all four handlers + %d-site "
-                       "sampling" % N_DRAWS if sample else args.workload + ": " + desc,
-                       "records_per_gpu": n, "sites": len(rec["sites"]),
-                       "threads": 32 * P.total_warps, "handlers": mask,
-                       "stored_bytes_per_gpu": 16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"],
-                       "algorithmic_bytes_per_gpu": alg_bytes,
-                       "l2": "inputs (%.1f GB) exceed the 126 MB L2; no flush" % (
-                           (16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"]) / 1e9),
-                       "parallelism": "dp%d (warp-id shards%s)" % (
-                           world, ", NCCL allreduce merge per step" if merge_on else "")},
-            "hbm_gbs": world * alg_bytes * args.steps / sec / 1e9,
-            "hbm_frac_of_spec_8tbs": alg_bytes * args.steps / sec / 1e9 / SPEC_HBM_GBS,
-            "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
-                         "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "peak_source": peak_src,
-                         "traffic": ncu_traffic(args.workload),
-                         "algorithmic_bytes_per_launch": alg_bytes,
-                         "consume_ms_avg": consume_avg_s * 1e3,
-                         "consume_share_of_step": (consume_avg_s * 1e3) / (ms / args.steps)},
-            "gpu_launches": launches,
-            "clocks": clk.result(),
-        }
-        if e2e:
-            line["e2e"] = e2e
-        if cpu:
-            line["cpu_baseline"] = cpu
-        if slow:
-            line["instrumented_slowdown"] = slow
-        if online:
-            line["online_trace"] = online
-        if inj:
-            line["error_injection"] = inj
-        print(json.dumps(line), flush=True)
-    if comm is not None:
-        sassi.sassi_nccl_comm_destroy(comm)
+    if own_comm is not None:
+        sassi.sassi_nccl_comm_destroy(own_comm)
     ctx.close()
-    if launched:
-        dist.destroy_process_group()
+    if rank != 0:
+        return None
+    stored = 16 * n + 256 * rec["n_addr_rows"] + 128 * rec["n_val_rows"]
+    line = {
+        "metric": METRIC, "value": value, "unit": "records/s", "n_gpus": world,
+        "steps": steps, "warmup": args.warmup, "ms_per_step": ms / steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic",
+        "config": {"workload": workload + ": " + desc + (", all four handlers + %d-site sampling" %
+                                                         N_DRAWS if sample else ""),
+                   "records_per_gpu": n, "sites": len(rec["sites"]),
+                   "threads": 32 * P.total_warps, "handlers": mask,
+                   "stored_bytes_per_gpu": stored, "algorithmic_bytes_per_gpu": alg_bytes,
+                   "l2": "inputs (%.1f GB) exceed the 126 MB L2; no flush" % (stored / 1e9),
+                   "parallelism": "dp%d (warp-id shards%s)" % (
+                       world, ", NCCL allreduce merge per step" if merge_on else "")},
+        "hbm_gbs": world * alg_bytes * steps / sec / 1e9,
+        "hbm_frac_of_spec_8tbs": alg_bytes * steps / sec / 1e9 / SPEC_HBM_GBS,
+        "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
+                     "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "peak_source": peak_src,
+                     "traffic": ncu_traffic(workload),
+                     "algorithmic_bytes_per_launch": alg_bytes,
+                     "consume_ms_avg": consume_avg_s * 1e3,
+                     "consume_share_of_step": (consume_avg_s * 1e3) / (ms / steps)},
+        "gpu_launches": launches,
+        "clocks": clk.result(),
+    }
+    for k, v in (("e2e", e2e), ("cpu_baseline", cpu), ("instrumented_slowdown", slow),
+                 ("online_trace", online), ("error_injection", inj)):
+        if v:
+            line[k] = v
+    return line
+
+
+def main():
+    args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(self_launch(args.gpus))
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        sys.exit("bench.py: --gpus %d but WORLD_SIZE=%d (launch one rank per GPU)" % (args.gpus, world))
+    if args.selftest_dist:
+        run_selftest_dist(args, rank, world)
+        return
+    args.workload = args.workload or ("c3" if world == 1 else "c5")
+    if args.impl == "reference":
+        run_reference(args, rank, world, args.workload)
+        return
+    import torch
+    import torch.distributed as dist
+    torch.cuda.set_device(local)
+    if "RANK" in os.environ:  # under torchrun (any world size)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    try:
+        if args.workload == "c5":
+            run_c5(args, rank, world, local)
+        else:
+            line = run_weak(args, rank, world, local, args.workload)
+            if line is not None:
+                print(json.dumps(line), flush=True)
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
 
 
 def measure_injection(dev, k=1000):

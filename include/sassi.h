@@ -257,7 +257,10 @@ int sassi_index_records(struct sassi_ctx* ctx, const sassi_hdr* hdr, uint64_t n,
 int sassi_reset(struct sassi_ctx* ctx, void* stream);
 
 /* Copy the table image (sassi_table_layout(...).total words) to HOST memory; synchronises
- * `stream` (CUPTI kernel-exit callback analogue, L217). Errors: EINVAL (n_words too small). */
+ * `stream` (CUPTI kernel-exit callback analogue, L217). Errors: EINVAL (n_words too small),
+ * EFORMAT (a consume since the last sassi_reset found the record stream inconsistent with its rows
+ * or chunk index: the tables are then incomplete), EMISMATCH (a sassi_merge found other site
+ * tables on another rank and left the tables unmerged). */
 int sassi_read_tables(struct sassi_ctx* ctx, uint64_t* host_out, uint64_t n_words, void* stream);
 
 /* Device pointer to the live table image (owned by the context; read-only for the caller). */
@@ -283,8 +286,22 @@ int sassi_sample_sites_device(struct sassi_ctx* ctx, uint32_t k, uint64_t seed,
  * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits); with
  * dynamic pcs enabled, also an ncclAllGather of every rank's dynamic table, which each rank
  * re-inserts into a cleared table (every rank then holds the same entries).
+ * A 2-word allreduce first compares the ranks' site-table checksums. The first merge of a context
+ * over a communicator (and every merge with dynamic pcs enabled) synchronises `stream` to check it
+ * on the host (EMISMATCH before any table traffic); later merges check it on the device with no
+ * host round trip: a mismatch then leaves the tables unmerged and the next sassi_read_tables
+ * returns EMISMATCH. A configuration change (sassi_select_memdiv_pcs, sassi_enable_dynamic_pcs)
+ * must be made identically on every rank.
  * Collective: every rank must call it. Errors: ENCCL, EMISMATCH (site tables differ). */
 int sassi_merge(struct sassi_ctx* ctx, void* nccl_comm, void* stream);
+
+/* The same merge for n contexts on ONE device (e.g. warp shards folded into separate contexts, or
+ * one context per stream): every context ends with the merged tables. It runs sassi_merge's pack
+ * and unpack kernels with the allreduce replaced by a device sum of the n packed images
+ * (isScalar / mask bytes compared with n), and merges dynamic-pc tables like sassi_merge.
+ * Stream-ordered, no host synchronisation. ctxs: HOST array of n distinct contexts (n <= 255) with
+ * identical site tables, warps and pc selections (EMISMATCH otherwise), all on one device (EINVAL). */
+int sassi_merge_local(struct sassi_ctx* const* ctxs, uint32_t n, void* stream);
 
 /* ---- Fused fold + merge over peer memory (one node: NVLink / NVSwitch P2P, or one device) ----
  * Instead of folding and then running sassi_merge's collective, every rank can fold straight into

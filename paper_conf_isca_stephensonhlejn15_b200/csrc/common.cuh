@@ -28,6 +28,10 @@ constexpr uint64_t kMaxRecordsPerLaunch = 1ull << 29;  // 32-bit record / row in
 constexpr uint32_t kDynLocalLg = 9, kDynLocal = 1u << kDynLocalLg;  // per-CTA dynamic-pc cache slots
 constexpr uint32_t kDynLocalWords = 4 * kDynLocal;                  // key + count (u32) + threads (u64)
 constexpr uint32_t kMaxPeers = 7;   // fused merge over peer memory: up to 8 GPUs of one node
+// error-flag bits (ctx->d_err, reported by sassi_read_tables): 4 = rows of a batch run past its
+// chunk's rows or the index disagrees with the rows, 8 = chunk index outside the row buffers
+// (both SASSI_EFORMAT); kMergeMismatch = a merge found other site tables (SASSI_EMISMATCH)
+constexpr uint32_t kErrRows = 4u, kErrIndex = 8u, kMergeMismatch = 1u << 16;
 
 // Packed per-site info word in the hash (bit layout). The companion cidx word holds the
 // site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).
@@ -162,6 +166,8 @@ struct sassi_ctx {
   // merge scratch
   uint64_t* d_pack = nullptr;
   uint64_t pack_words = 0;
+  void* verified_comm = nullptr;     // communicator whose ranks were proven to hold this layout ...
+  uint64_t verified_checksum = 0;   // ... for this checksum (sassi_merge's host-synchronised check)
   // dynamic sites: insert-on-miss table of unregistered pcs (sassi_enable_dynamic_pcs)
   uint32_t dyn_cap = 0, dyn_lg = 0;
   uint32_t* d_dyn_keys = nullptr;           // [dyn_cap]
@@ -196,6 +202,7 @@ int launch_sample(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* host_
 int launch_sample_device(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* dev_out,
                          uint32_t* dev_status, cudaStream_t s);
 int launch_merge(sassi_ctx* c, void* comm, cudaStream_t s);
+int launch_merge_local(sassi_ctx* const* ctxs, uint32_t n, cudaStream_t s);
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes);
 int launch_dyn_reset(sassi_ctx* c, cudaStream_t s);
 

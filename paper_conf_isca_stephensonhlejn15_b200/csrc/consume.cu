@@ -16,8 +16,8 @@
 //                                  category totals are formed at the flush
 // Work split: a warp owns one 256-record chunk at a time (chunk_base gives its row offsets) and walks
 // it in 8 batches of 32 records; row indices inside a batch come from ballot prefix sums.
+#include <map>
 #include <mutex>
-#include <unordered_map>
 #include <utility>
 
 #include "common.cuh"
@@ -326,15 +326,17 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   unsigned long long* const table = reinterpret_cast<unsigned long long*>(p.table);
   // every table update goes to this context's image and to the peers' (fused merge: the atomics
   // travel over NVLink to the other GPUs' images, so no collective runs after the fold)
+  // (peer images live on other GPUs: system-scope atomics, atom.sys, so that updates from several
+  // GPUs to one word are atomic with each other; the own image keeps device scope)
   auto gadd = [&](uint64_t off, unsigned long long v) {
     atomicAdd(table + off, v);
     if (kExt)
-      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAdd(p.peers[j] + off, v);
+      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAdd_system(p.peers[j] + off, v);
   };
   auto gand = [&](uint64_t off, unsigned long long v) {
     atomicAnd(table + off, v);
     if (kExt)
-      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd(p.peers[j] + off, v);
+      for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd_system(p.peers[j] + off, v);
   };
 
   // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239). Returns the
@@ -487,7 +489,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     const ulonglong2 cb1 = kUnitRows ? p.cb[u + 1] : cb0;
     if (kUnitRows && !(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end &&
                        cb0.y >= p.vrow_base && cb0.y <= cb1.y && cb1.y <= p.vrow_end)) {
-      err |= 8u;  // chunk index outside the row buffers
+      err |= kErrIndex;  // chunk index outside the row buffers
       continue;
     }
     // rows are addressed relative to this chunk: 32-bit offsets from here on
@@ -530,7 +532,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
         arow += __popc(ma);
         vrow += vtot;
         if (arow > aend || vrow > vend) {
-          err |= 4u;  // rows of this batch run past the chunk's rows: stream inconsistent
+          err |= kErrRows;  // rows of this batch run past the chunk's rows: stream inconsistent
           break;
         }
       }
@@ -666,7 +668,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       }
     }
     if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && lane == 0 && (arow != aend || vrow != vend))
-      err |= 4u;  // index disagrees with the rows
+      err |= kErrRows;  // index disagrees with the rows
   }
   if (H & SASSI_H_INSTCOUNT) {
     if (kVertical) flush_planes();
@@ -830,11 +832,12 @@ int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
   if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
   if ((void*)fn != c->launch_fn || c->smem_bytes != c->launch_smem) {  // configure once per kernel
     {
-      // the attribute is per function and process-wide: only ever raise it (contexts share kernels)
+      // the attribute is per function and per device (CUDA context): only ever raise it, keyed on
+      // (device, function) since contexts on one device share kernels
       static std::mutex mu;
-      static std::unordered_map<void*, size_t> attr;
+      static std::map<std::pair<int, void*>, size_t> attr;
       std::lock_guard<std::mutex> lock(mu);
-      size_t& cur = attr[(void*)fn];
+      size_t& cur = attr[{c->device, (void*)fn}];
       if (c->smem_bytes > cur) {
         SASSI_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c->smem_bytes));
         cur = c->smem_bytes;

@@ -58,6 +58,7 @@ SIGNATURES = {
     "sassi_sample_sites": (_i, [_vp, _u32, _u64, _vp, _vp]),
     "sassi_sample_sites_device": (_i, [_vp, _u32, _u64, _vp, _vp, _vp]),
     "sassi_merge": (_i, [_vp, _vp, _vp]),
+    "sassi_merge_local": (_i, [_vp, _u32, _vp]),
     "sassi_nccl_get_unique_id": (_i, [_vp]),
     "sassi_nccl_comm_create": (_i, [ctypes.POINTER(_vp), _i, _i, _vp, _i]),
     "sassi_nccl_comm_destroy": (_i, [_vp]),
@@ -223,6 +224,12 @@ def sassi_sample_sites_device(ctx: int, k: int, seed: int, dev_out: int, dev_sta
 
 def sassi_merge(ctx: int, comm: int, stream=None) -> None:
     _check(lib().sassi_merge(ctx, comm, _stream(stream)))
+
+
+def sassi_merge_local(ctxs, stream=None) -> None:
+    """Merge n contexts of one device in place (each ends with the merged tables)."""
+    arr = (_vp * len(ctxs))(*[getattr(c, "handle", c) for c in ctxs])
+    _check(lib().sassi_merge_local(arr, len(ctxs), _stream(stream)))
 
 
 def sassi_nccl_get_unique_id() -> bytes:

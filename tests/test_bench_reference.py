@@ -1,6 +1,9 @@
 """bench.py --impl reference (the oracle timed on the host, the driver's reference arm) keeps the
 JSON contract on a CPU-only host: one line with the metric, a positive value, cpu_baseline and e2e
-describing the run; under torchrun with two ranks only rank 0 prints (the others exit 0)."""
+describing the run; under torchrun with two ranks only rank 0 prints (the others exit 0). The N > 1
+workload is c5 (the configuration the metric quotes for 8 GPUs). `bench.py --gpus 2` without
+torchrun launches the two ranks itself (self-launch), and the distributed plumbing (gloo on a CPU
+host: rendezvous, barrier, max over ranks) prints one line with n_gpus = 2."""
 import json
 import os
 import socket
@@ -14,13 +17,13 @@ def _lines(out):
     return [json.loads(l) for l in out.splitlines() if l.startswith("{")]
 
 
-def _check(d):
+def _check(d, workload="c3"):
     assert d["impl"] == "reference" and d["unit"] == "records/s" and d["value"] > 0
     assert d["metric"].startswith("warp-instr records/sec") and d["higher_is_better"] is True
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert abs(d["cpu_baseline"]["value"] - d["value"]) < 1e-6 * d["value"]
     assert d["e2e"]["value"] == d["value"] and d["e2e"]["h2d_bytes_per_step"] == 0
-    assert d["config"]["workload"].startswith("c3")
+    assert d["config"]["workload"].startswith(workload)
 
 
 def test_reference_arm_single_process():
@@ -45,5 +48,39 @@ def test_reference_arm_under_torchrun_prints_once():
     assert r.returncode == 0, r.stderr[-2000:]
     lines = _lines(r.stdout)
     assert len(lines) == 1
-    _check(lines[0])
-    assert lines[0]["n_gpus"] == 2
+    _check(lines[0], "c5")
+    assert lines[0]["n_gpus"] == 2 and lines[0]["scaling"] == "strong"
+
+
+def test_gpus_flag_self_launches_reference_arm():
+    """`bench.py --gpus 2` outside torchrun re-launches itself with two ranks."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference",
+                        "--gpus", "2", "--steps", "1", "--warmup", "0"], capture_output=True,
+                       text=True, timeout=600, cwd=ROOT, env={k: v for k, v in os.environ.items()
+                                                             if k not in ("RANK", "WORLD_SIZE")})
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _lines(r.stdout)
+    assert len(lines) == 1 and lines[0]["n_gpus"] == 2
+    _check(lines[0], "c5")
+    assert lines[0]["cpu_baseline"]["nproc"] >= 1 and lines[0]["cpu_baseline"]["threads"] == 1
+
+
+def test_gpus_flag_self_launches_dist_plumbing():
+    """The multi-rank plumbing of the bench (process group, barrier, max-over-ranks) with gloo on
+    this CPU host: one line from rank 0 with n_gpus = 2 and both ranks reporting."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--selftest-dist", "--gpus", "2"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT,
+                       env={k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE")})
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _lines(r.stdout)
+    assert len(lines) == 1
+    d = lines[0]
+    assert d["n_gpus"] == 2 and d["ranks_reporting"] == 2 and d["backend"] in ("gloo", "nccl")
+    assert d["max_over_ranks_s"] >= 0.02        # rank 1 sleeps 20 ms: the maximum is rank 1's
+
+
+def test_gpus_flag_must_match_world_size():
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--selftest-dist", "--gpus", "2"],
+                       capture_output=True, text=True, timeout=120, cwd=ROOT, env=env)
+    assert r.returncode != 0 and "WORLD_SIZE" in r.stderr
