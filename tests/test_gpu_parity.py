@@ -1,7 +1,8 @@
 """GPU parity: the CUDA fold (through the C ABI) equals the oracle bit for bit — hand-worked T0,
-random edge-case traces for every handler combination, and every BASELINE config (c1, c2 in
-full; c3/c4/c5 at full size in the bench's launch configuration, checked exactly on prefixes /
-sampled warps the oracle computes one by one, and by properties that hold at any size)."""
+random edge-case traces for every handler combination, and every BASELINE config in full: c1 and
+c2 with a single oracle pass; c3 and c4 (10^8 records) and one whole c5 shard (~4.9x10^8 records)
+in the bench's launch configuration, against the oracle run over host-generated warp shards in
+parallel processes and merged (tests/oracle_shards.py), plus properties that hold at any size."""
 import numpy as np
 import pytest
 
@@ -156,22 +157,21 @@ def _properties(sec, n):
 
 
 @pytest.mark.parametrize("name", ["c3", "c4"])
-def test_full_size_prefix_exact_and_properties(name):
-    """10^8 records in the bench's launch configuration: the whole stream is folded on the GPU;
-    its first ~2x10^6 records are checked bit-exactly against the oracle, the full tables by
-    invariants, and consuming the stream in two pieces equals consuming it at once."""
+def test_full_size_exact_and_properties(name):
+    """10^8 records in the bench's launch configuration: the whole stream folded on the GPU equals
+    the oracle over the whole stream in every table section (the oracle runs over host-generated
+    warp shards in parallel processes, merged with its own merge: tests/oracle_shards.py); the
+    invariants hold, and consuming the stream in two pieces equals consuming it at once."""
+    from oracle_shards import oracle_full
     P, mask, d = _gen(name)
     assert d["n"] == 100_000_000
     S, W = len(d["sites"]), P.total_warps
     full = gpu_table(d["sites"], W, mask, d)
     sec = oracle.sections(full, S, W)
     _properties(sec, d["n"])
-    # exact on a prefix
-    pre = _prefix(d, 2_000_128)
-    hp = gen.to_host(pre)
-    o = oracle.run(hp["sites"], W, mask, hp["hdr"], hp["addr"], hp["val"])
-    t = gpu_table(d["sites"], W, mask, pre)
-    assert diff_tables(t, o, S, W) is None
+    o, n = oracle_full(name, mask, limit=d["n"])
+    assert n == d["n"]
+    assert diff_tables(full, o, S, W) is None
     # split consumption == single pass (chunk-aligned split; rows addressed absolutely)
     ctx = sassi.Context(d["sites"], W, mask)
     half = (d["n"] // 2) // 256 * 256
@@ -365,11 +365,12 @@ def test_merge_single_rank_nccl():
     assert np.array_equal(after, oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val, pcs=sel))
 
 
-def test_c5_full_shard_sampled_warps_exact():
+def test_c5_full_shard_exact():
     """One full c5 shard (16,384 warps, ~4.9x10^8 records, ~90 GB in HBM) folded in the bench's
-    launch configuration. Per-thread counts are warp-disjoint, so the oracle computes them exactly
-    for sampled warps from those warps' records alone; the per-PC tables are checked by invariants
-    and by splitting the shard in two folds that accumulate to the single pass."""
+    launch configuration equals the oracle over the whole shard in every table section (parallel
+    host oracle over warp sub-shards, merged); the per-PC tables also satisfy the invariants and
+    two chunk-aligned halves accumulate to the single pass."""
+    from oracle_shards import oracle_full
     P, _, mask, _ = gen.preset("c5")
     W = P.total_warps
     shard = 3
@@ -379,19 +380,9 @@ def test_c5_full_shard_sampled_warps_exact():
     full = gpu_table(d["sites"], W, mask, d)
     sec = oracle.sections(full, S, W)
     _properties(sec, d["n"])
-    offs = np.zeros((16385, 3), np.uint64)
-    offs[1:] = np.cumsum(d["counts"], axis=0)
-    rng = np.random.default_rng(5)
-    for wl in sorted(rng.choice(16384, 6, replace=False).tolist()) + [0, 16383]:
-        r0, a0, v0 = (int(x) for x in offs[wl])
-        r1, a1, v1 = (int(x) for x in offs[wl + 1])
-        hdr = d["hdr"][r0:r1].cpu().numpy().view(np.uint32).reshape(-1, 4).view(gen.HDR_DTYPE).reshape(-1)
-        addr = d["addr"][a0:a1].cpu().numpy().view(np.uint64).reshape(-1, 32)
-        val = d["val"][v0:v1].cpu().numpy().view(np.uint32).reshape(-1, 32)
-        o = oracle.run(d["sites"], W, mask, hdr, addr, val)
-        gw = shard * 16384 + wl
-        so = oracle.sections(o, S, W)
-        assert np.array_equal(sec["counts"][32 * gw:32 * gw + 32], so["counts"][32 * gw:32 * gw + 32]), gw
+    o, n = oracle_full("c5", mask, warp_base=shard * 16384, n_warps=16384, warps_per_job=512)
+    assert n == d["n"]
+    assert diff_tables(full, o, S, W) is None
     # two chunk-aligned halves accumulate to the single pass
     half = (d["n"] // 2) // 256 * 256
     ctx = sassi.Context(d["sites"], W, mask)
