@@ -1,7 +1,9 @@
 """Error injection on the instrumented kernels (§8.1):
-profile -> draw sites -> one injection run per site. The injected instruction, register value and
-bit of every run equal what the oracle locates in the same kernel's trace (the dyn-th eligible,
-not-predicated-out dynamic instruction of the thread, reading R23); outcomes follow their rules."""
+profile -> draw sites -> one injection run per site. The injected instruction, target kind (a GPR
+destination chosen by reg_seed % n_gpr_dst, the stored word, the written predicate or one of the 4
+condition-code bits, L621 / L629), register value and bit of every run equal what the oracle
+locates in the same kernel's trace (the dyn-th eligible, not-predicated-out dynamic instruction of
+the thread, reading R23); outcomes follow their rules."""
 import numpy as np
 import pytest
 
@@ -12,6 +14,10 @@ pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
 SMALL = {"vecadd": 12800, "bfs": 4096, "sgemm": 64, "stencil": 64}
+TARGET_CODE = {"gpr": 0, "mem": 1, "pred": 2, "cc": 3}
+# target kinds a campaign reaches: vecadd has GPR (1 and 2 destinations), stores, a predicate and a
+# condition-code site; bfs and stencil a predicate site; sgemm GPRs and stores only
+EXPECTED_KINDS = {"vecadd": {0, 1, 2, 3}, "bfs": {0, 1, 2}, "sgemm": {0, 1}, "stencil": {0, 1, 2}}
 # the global stores into the kernels' outputs (a flipped stored word is always visible)
 OUTPUT_STORES = {"vecadd": {3}, "bfs": {8}, "sgemm": {9}, "stencil": {7}}
 
@@ -37,10 +43,46 @@ def test_injection_targets_equal_oracle_locate(name):
         assert loc is not None
         assert int(o["site"]) == loc["site"]
         assert int(o["bit"]) == loc["bit"]
-        assert int(o["target"]) == {"gpr": 0, "mem": 1}[loc["target"]]
-        if loc["target"] == "gpr":
+        assert int(o["target"]) == TARGET_CODE[loc["target"]]
+        if loc["target"] == "gpr":   # the chosen destination's value (reg_seed % n_gpr_dst)
             assert int(o["before"]) == loc["before"]
+        if loc["target"] == "pred":
+            assert int(o["before"]) in (0, 1) and int(o["bit"]) == 0
+        if loc["target"] == "cc":
+            assert int(o["before"]) < 16 and int(o["bit"]) < 4
         assert int(o["after"]) == int(o["before"]) ^ (1 << int(o["bit"]))
+    kinds = set(int(t) for t in outs["target"])
+    assert kinds == EXPECTED_KINDS[name], kinds
+    ik.close()
+
+
+def test_injection_two_destination_choice():
+    """vecadd's IMAD.WIDE site (s8) writes R4:R5: reg_seed picks the destination (L629), so the
+    flipped value is the low or the high half of the 64-bit address, as the oracle locates."""
+    ik = sassi.InstrumentedKernel("vecadd", SMALL["vecadd"])
+    ctx = ik.context(sassi.SASSI_H_INSTCOUNT)
+    rec = ik.trace(ctx)
+    ctx.close()
+    h = gen.to_host(rec)
+    s8 = [i for i, r in enumerate(h["hdr"]) if r["pc"] == h["sites"][8]["pc"] and r["warp"] == 0][0]
+    # thread 0's eligible instructions before its first s8 record: count them from the trace
+    dyn = sum(1 for r in h["hdr"][:s8] if r["warp"] == 0 and r["pc"] in h["sites"]["pc"] and
+              (h["sites"][list(h["sites"]["pc"]).index(r["pc"])]["n_gpr_dst"] > 0 or
+               h["sites"][list(h["sites"]["pc"]).index(r["pc"])]["flags"] & (gen.F_MEM | gen.F_WRITES_PRED | gen.F_WRITES_CC))
+              and (r["active"] & r["mask2"]) & 1)
+    st = np.zeros(2, dtype=sassi.INJ_DTYPE)
+    st["thread"] = 0
+    st["dyn_index"] = dyn
+    st["reg_seed"] = [4, 7]                         # destination 0 (low half), then 1 (high half)
+    st["bit_seed"] = [3, 3]
+    outs = ik.inject(st)
+    for t, o in zip(st, outs):
+        loc = oracle.locate_injection(h["sites"], h["hdr"], h["val"], 0, dyn, int(t["reg_seed"]), 3)
+        assert loc["site"] == 8 == int(o["site"]) and loc["target"] == "gpr"
+        assert int(o["before"]) == loc["before"]
+    assert int(outs["before"][0]) != int(outs["before"][1])   # the two halves of the address
+    # a flipped high-half bit sends the load far outside A: the crash symptom (DUE)
+    assert int(outs["outcome"][1]) == sassi.SASSI_INJ_DUE
     ik.close()
 
 
@@ -56,9 +98,17 @@ def test_injection_outcome_rules(name):
     # a flipped word stored to the output is always an SDC
     stores = np.isin(outs["site"], list(OUTPUT_STORES[name]))
     assert stores.any() and (oc[stores] == sassi.SASSI_INJ_SDC).all()
-    # only the kernel with data-dependent indices and trip counts shows crash / hang symptoms
+    # hangs need data-dependent trip counts (bfs); crashes need a corruptible address or index:
+    # bfs indices, vecadd's 64-bit addresses (IMAD.WIDE / IADD.CC carry), stencil's border points
+    # reached through a flipped predicate; sgemm has neither
     if name != "bfs":
-        assert not np.isin(oc, [sassi.SASSI_INJ_DUE, sassi.SASSI_INJ_HANG]).any()
+        assert not (oc == sassi.SASSI_INJ_HANG).any()
+    if name == "sgemm":
+        assert not (oc == sassi.SASSI_INJ_DUE).any()
+    # a flipped predicate or condition code changes control or the address, or nothing (masked)
+    pcc = np.isin(outs["target"], [2, 3])
+    if pcc.any():
+        assert np.isin(oc[pcc], [sassi.SASSI_INJ_MASKED, sassi.SASSI_INJ_SDC, sassi.SASSI_INJ_DUE]).all()
     # the same tuples give the same outcomes, and the outputs are left error-free
     again = ik.inject(sites)
     assert np.array_equal(again, outs)

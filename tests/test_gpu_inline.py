@@ -102,9 +102,9 @@ def test_instrumented_vecadd_is_config_c1():
     for s in (0, 1, 3):
         assert list(map(int, sec["mem"][s])) == [400, 12800, 1600, 400]
     assert list(map(int, sec["mem"][5])) == [400, n3, n3, n3]
-    # per-thread counts: 6 eligible sites per iteration (2 LDG, FADD, STG) + the x load and the
-    # running sum in iterations where i % 3 == 0
-    expect = 4 * 100 + 2 * np.array([sum(1 for it in range(100) if (128 * it + t) % 3 == 0)
+    # per-thread counts: 7 eligible sites per iteration (IMAD.WIDE, IADD.CC, 2 LDG, FADD, STG,
+    # ISETP) + the x load and the running sum in iterations where i % 3 == 0
+    expect = 7 * 100 + 2 * np.array([sum(1 for it in range(100) if (128 * it + t) % 3 == 0)
                                       for t in range(128)])
     assert np.array_equal(sec["counts"].astype(np.int64), expect)
     ctx.close()
