@@ -99,7 +99,7 @@ typedef struct sassi_ctx sassi_ctx;
 #define SASSI_ABI_VERSION 3u
 #define SASSI_WARP_SIZE 32u
 #define SASSI_CHUNK 256u           /* records per chunk_base entry */
-#define SASSI_MAX_SITES 4096u      /* registered sites per context */
+#define SASSI_MAX_SITES 65536u     /* registered sites per context (beyond ~4k: global mode, see attach) */
 #define SASSI_MAX_DST 4u           /* GPR destinations per instruction (e.g. 128-bit loads) */
 #define SASSI_MAX_PC_MATRICES 4u   /* per-PC memdiv matrices (sassi_select_memdiv_pcs)          */
 
@@ -195,7 +195,12 @@ void sassi_ctx_destroy(struct sassi_ctx* ctx);
 
 /* Select which handlers run (non-empty subset of SASSI_H_EVERY) — the paper's "what"
  * (L181-L187). Allowed only before the first consume or right after sassi_reset, and not to a
- * different set while peer tables are attached. Errors: EINVAL, ESTATE, ENOSPC. */
+ * different set while peer tables are attached. The fold keeps the pc hash, the value state and
+ * the per-site counters in each SM's shared memory when they fit; a larger site table (thousands
+ * of sites, up to SASSI_MAX_SITES) runs in "global mode": hash lookups from global memory and
+ * per-record u64 atomics into the table image (the paper's own device-global tables),
+ * same results, lower throughput. Errors: EINVAL, ESTATE, ENOSPC (the 32x32 matrices and the
+ * per-PC matrices alone exceed shared memory: not reachable with SASSI_MAX_PC_MATRICES). */
 int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
 
 /* Keep a per-PC memory-divergence matrix (pcmat, the Fig.6 32x32 matrix of that pc's own records)

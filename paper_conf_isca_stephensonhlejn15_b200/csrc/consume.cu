@@ -254,8 +254,13 @@ uint32_t sm_var_words(uint32_t H) {
 }
 
 // kExt: the extended instantiation, used when the insert-on-miss table of unregistered pcs is
-// enabled (p.dyn_cap) and / or the flush also updates peers' images (p.n_peers); the plain kernels
-// carry none of that code
+// enabled (p.dyn_cap), the flush also updates peers' images (p.n_peers), and / or the site table
+// does not fit shared memory (p.gmode: the "global mode" below); the plain kernels carry none of it.
+// Global mode (site tables beyond one SM's shared memory, up to SASSI_MAX_SITES): the pc hash is
+// read from global memory (L1 / L2 resident), each record's counters are added straight to the u64
+// table image with device atomics (Fig.4 / Fig.9's own atomicAdd / atomicAnd into a device-global
+// table, L239 / L595), and the value state is ANDed into the image's constantOnes / constantZeros /
+// isScalar words when a bit changes; only the 32x32 matrices stay in shared memory.
 template <uint32_t H, bool kExt>
 __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const ConsumeParams p) {
   extern __shared__ __align__(128) uint32_t sm[];
@@ -264,11 +269,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
                      kSmBar = Ly::kBar, kSmVbuf = Ly::kVbuf, kSmVar = Ly::kVar;
   constexpr uint32_t kCounters = SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX;
   const uint32_t cap = p.cap;
+  const bool gm = kExt && p.gmode;  // global mode: no hash, value state or counters in smem
+  const uint32_t scap = gm ? 0u : cap;
   uint4* s_hash = reinterpret_cast<uint4*>(sm + kSmVar);            // [cap] {key, info, cidx, -}
-  uint4* s_vstate = s_hash + cap;                                   // [nvd] ones, zeros, isScalar
-  uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + (Ly::kVal ? p.nvd : 0u));  // counters
+  uint4* s_vstate = s_hash + scap;                                  // [nvd] ones, zeros, isScalar
+  uint32_t* s_priv = reinterpret_cast<uint32_t*>(s_vstate + (Ly::kVal && !gm ? p.nvd : 0u));  // counters
   // [npcm][32][32] per-PC matrices (the private counters exist only for handler sets that count)
-  uint32_t* s_pcm = s_priv + ((H & kCounters) ? (p.priv ? kWarpsPerCta : 1u) * p.pw : 0u);
+  uint32_t* s_pcm = s_priv + ((H & kCounters) && !gm ? (p.priv ? kWarpsPerCta : 1u) * p.pw : 0u);
   // dynamic sites: a per-CTA insert-on-miss cache of unregistered pcs (keys, record counts, thread
   // counts), flushed into the global table at CTA exit
   uint32_t* const s_dkey = s_pcm + 1024 * p.npcm;
@@ -277,10 +284,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
 
   const uint32_t tid = threadIdx.x;
-  for (uint32_t i = tid; i < cap; i += blockDim.x) s_hash[i] = p.hash[i];
-  if (Ly::kVal)
+  for (uint32_t i = tid; i < scap; i += blockDim.x) s_hash[i] = p.hash[i];
+  if (Ly::kVal && !gm)
     for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
-  if (H & kCounters)
+  if ((H & kCounters) && !gm)
     for (uint32_t i = tid; i < n_regions * p.pw; i += blockDim.x) s_priv[i] = 0;
   for (uint32_t i = tid; i < kSmBar; i += blockDim.x) sm[i] = 0;  // diag (+ matrices)
   if (H & SASSI_H_MEMDIV)
@@ -339,16 +346,27 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       for (uint32_t j = 0; j < p.n_peers; ++j) atomicAnd_system(p.peers[j] + off, v);
   };
 
+  // global mode: this lane's record adds v.x.. to the u64 words base + 0.. of the image
+  auto gcount4 = [&](bool pred, uint64_t base, uint4 v) {
+    if (pred) {
+      gadd(base, (unsigned long long)v.x);
+      if (v.y) gadd(base + 1, (unsigned long long)v.y);
+      if (v.z) gadd(base + 2, (unsigned long long)v.z);
+      if (v.w) gadd(base + 3, (unsigned long long)v.w);
+    }
+  };
+  unsigned long long g_imix[7] = {0, 0, 0, 0, 0, 0, 0};  // global mode: Fig.3 totals of this warp
+
   // ---- find(pc): open-addressed, linear probing, one 16-byte slot per probe (L239). Returns the
   // slot {key, info, cidx, site}; `known` = a registered site (0xFFFFFFFF is never registered) ----
   // h is always a real header of the stream (loads are clamped), so the probe needs no guard;
   // records are counted per chunk / range (c_rec), not here
   auto lookup = [&](const uint4& h, bool valid, bool& known) -> uint4 {
     uint32_t slot = pc_slot(h.x, p.hmul, p.hshr, cap);
-    uint4 e = s_hash[slot];
+    uint4 e = gm ? __ldg(p.hash + slot) : s_hash[slot];
     while (e.x != h.x && e.x != EMPTY_KEY) {  // collision: linear probing (load <= 1/2, rare)
       slot = (slot + 1) & (cap - 1);
-      e = s_hash[slot];
+      e = gm ? __ldg(p.hash + slot) : s_hash[slot];
     }
     known = valid && e.x == h.x && h.x != EMPTY_KEY;
     c_unk += valid && !known;
@@ -386,14 +404,30 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     // ---- Case study I: branch divergence (Fig.4) ----
     if (H & SASSI_H_BRANCH) {
       const bool isb = live && (info & I_BRANCH);
-      add_counters4(isb, 4 * (cidx & 0xFFFFu),
-                    make_uint4(1u, (uint32_t)__popc(act), (uint32_t)__popc(G),
-                               (G != 0 && G != act) ? 1u : 0u),
-                    wpriv);
+      const uint32_t na = __popc(act), nt = __popc(G);
+      const uint32_t dv = (G != 0 && G != act) ? 1u : 0u;
+      if (gm) {
+        if (isb) {
+          gadd(p.off.br + 5ull * site, 1ull);
+          gadd(p.off.br + 5ull * site + 1, (unsigned long long)na);
+          if (nt) gadd(p.off.br + 5ull * site + 2, (unsigned long long)nt);
+          if (na - nt) gadd(p.off.br + 5ull * site + 3, (unsigned long long)(na - nt));
+          if (dv) gadd(p.off.br + 5ull * site + 4, 1ull);
+        }
+      } else {
+        add_counters4(isb, 4 * (cidx & 0xFFFFu), make_uint4(1u, na, nt, dv), wpriv);
+      }
     }
     // ---- Fig.3 instruction mix (L193-L199): every active thread counts; per-site thread
     // executions here, the seven category totals at the flush (R22) ----
-    if ((H & SASSI_H_INSTMIX) && live) atomicAdd(wpriv + p.px + site, (uint32_t)__popc(act));
+    if ((H & SASSI_H_INSTMIX) && !gm && live) atomicAdd(wpriv + p.px + site, (uint32_t)__popc(act));
+    if ((H & SASSI_H_INSTMIX) && gm) {  // global mode: the site's word and the categories per batch
+      const uint32_t np = live ? (uint32_t)__popc(act) : 0u;
+      if (np) gadd(p.off.mix + site, (unsigned long long)np);
+      const uint32_t cat = live ? __ldg(p.flush_x + site) : 0u;
+#pragma unroll
+      for (uint32_t k = 0; k < 7; ++k) g_imix[k] += __reduce_add_sync(FULL, ((cat >> k) & 1u) ? np : 0u);
+    }
     // ---- Case study IV: per-thread eligible dynamic-instruction counts (§8.1) ----
     if (H & SASSI_H_INSTCOUNT) {
       uint32_t E = (live && (info & I_ELIGIBLE)) ? G : 0u;
@@ -603,16 +637,25 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
             if (info & I_PCM)  // this pc's own matrix (sassi_select_memdiv_pcs)
               atomicAdd(s_pcm + 1024 * ((info >> I_PCM_SHIFT) & 3u) + 32 * (n - 1) + (my_s - 1), 1u);
           }
-          add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv);
+          if (gm) gcount4(selm_l, p.off.mem + 4ull * e.w, make_uint4(1u, n, my_s, my_l));
+          else add_counters4(selm_l, PB + 4 * (cidx & 0xFFFFu), make_uint4(1u, n, my_s, my_l), wpriv);
         }
       }
       // ---- Case study III: value profiling (Fig.9): row-per-lane fold of TMA-staged rows ----
       if (H & SASSI_H_VALUE) {
         const bool selv = live && nd > 0 && G != 0;
-        add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv);
+        if (gm) {
+          if (selv) {
+            gadd(p.off.val + 2ull * e.w, 1ull);
+            gadd(p.off.val + 2ull * e.w + 1, (unsigned long long)__popc(G));
+          }
+        } else {
+          add_counters2(selv, PV + 2 * (cidx >> 16), make_uint2(1u, (uint32_t)__popc(G)), wpriv);
+        }
         if (vtot) {
           const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
-          const uint32_t vslot = (info >> I_VD0_SHIFT) & 0xFFFFu;  // its first value-state slot
+          // its first value-state slot (global mode: 4 * site, the image's [S][4] words)
+          const uint32_t vslot = gm ? 4u * e.w : (info >> I_VD0_SHIFT) & 0xFFFFu;
           for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
             const uint32_t nr = min(vtot - s0, 32u);
             if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
@@ -654,13 +697,20 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
                 vo |= (x.x & m0) | (x.y & m1) | (x.z & m2_) | (x.w & m3);
               }
             }
-            if (V != 0) {
+            if (V != 0 && !gm) {
               uint4* st = s_vstate + slot;
               const uint4 c = *st;
               const uint32_t sc = va == vo ? 1u : 0u;                  // __all(v == leader) (L559)
               if ((c.x & va) != c.x) atomicAnd(&st->x, va);           // constantOnes   (L557)
               if ((c.y & ~vo) != c.y) atomicAnd(&st->y, ~vo);         // constantZeros  (L557)
               if ((c.z & sc) != c.z) atomicAnd(&st->z, sc);           // isScalar       (L561)
+            } else if (V != 0) {  // global mode: the image's words (a stale read only adds an AND)
+              const uint32_t cx = (uint32_t)__ldcg(table + p.off.ones + slot);
+              const uint32_t cy = (uint32_t)__ldcg(table + p.off.zeros + slot);
+              const uint32_t cz = (uint32_t)__ldcg(table + p.off.scalar + slot);
+              if ((cx & va) != cx) gand(p.off.ones + slot, (unsigned long long)va);
+              if ((cy & ~vo) != cy) gand(p.off.zeros + slot, (unsigned long long)(uint32_t)~vo);
+              if (cz && va != vo) gand(p.off.scalar + slot, 0ull);
             }
           }
           __syncwarp();
@@ -707,7 +757,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     }
     return t;
   };
-  if (H & SASSI_H_BRANCH) {
+  if ((H & SASSI_H_BRANCH) && !gm) {
     for (uint32_t bi = tid; bi < p.nb; bi += blockDim.x) {
       const uint4 t = sum_words(4 * bi);
       if (t.x == 0) continue;
@@ -720,7 +770,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     }
   }
   if (H & SASSI_H_MEMDIV) {
-    for (uint32_t m = tid; m < p.nm; m += blockDim.x) {
+    for (uint32_t m = tid; !gm && m < p.nm; m += blockDim.x) {
       const uint4 t = sum_words(PB + 4 * m);
       if (t.x == 0) continue;
       const uint64_t g = p.off.mem + 4ull * p.flush_m[m];
@@ -738,7 +788,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   }
   if (H & SASSI_H_INSTMIX) {
     unsigned long long* const s_imix = reinterpret_cast<unsigned long long*>(sm + kSmImix);
-    for (uint32_t st = tid; st < p.S; st += blockDim.x) {
+    if (gm && lane == 0)  // global mode: the warps' Fig.3 totals
+      for (uint32_t k = 0; k < 7; ++k)
+        if (g_imix[k]) atomicAdd(s_imix + k, g_imix[k]);
+    for (uint32_t st = tid; !gm && st < p.S; st += blockDim.x) {
       uint32_t t = 0;
       for (uint32_t w = 0; w < n_regions; ++w) t += s_priv[w * p.pw + p.px + st];
       if (t == 0) continue;
@@ -750,7 +803,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     __syncthreads();
     if (tid < 7 && s_imix[tid]) gadd(p.off.imix + tid, s_imix[tid]);
   }
-  if (H & SASSI_H_VALUE) {
+  if ((H & SASSI_H_VALUE) && !gm) {
     for (uint32_t k = tid; k < p.nv; k += blockDim.x) {
       const uint32_t site = p.flush_v[3 * k], vd0 = p.flush_v[3 * k + 1], nd = p.flush_v[3 * k + 2];
       uint32_t we = 0, te = 0;
@@ -817,10 +870,13 @@ int launch_dyn_reset(sassi_ctx* c, cudaStream_t s) {
 
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
   const uint32_t H = c->mask;
-  size_t words = sm_var_words(H) + 4ull * c->cap;
-  if (H & SASSI_H_VALUE) words += 4ull * c->nvd;
-  if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX))
-    words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
+  size_t words = sm_var_words(H);
+  if (!c->gmode) {  // global mode keeps the hash, the value state and the counters in global memory
+    words += 4ull * c->cap;
+    if (H & SASSI_H_VALUE) words += 4ull * c->nvd;
+    if (H & (SASSI_H_BRANCH | SASSI_H_MEMDIV | SASSI_H_VALUE | SASSI_H_INSTMIX))
+      words += (c->priv ? kWarpsPerCta : 1) * (size_t)c->pw;
+  }
   if (H & SASSI_H_MEMDIV) words += 1024ull * c->npcm;  // per-PC matrices
   if (c->dyn_cap) words += kDynLocalWords;              // the CTA's dynamic-pc cache
   *bytes = 4 * words;
@@ -828,7 +884,7 @@ int consume_smem_bytes(const sassi_ctx* c, size_t* bytes) {
 }
 
 int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
-  KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0 || p.n_peers != 0);
+  KernelFn fn = select_kernel(c->mask, p.dyn_cap != 0 || p.n_peers != 0 || p.gmode != 0);
   if (!fn) return set_error(SASSI_ESTATE, "no handler attached");
   if ((void*)fn != c->launch_fn || c->smem_bytes != c->launch_smem) {  // configure once per kernel
     {
