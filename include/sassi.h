@@ -212,6 +212,16 @@ int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
  * Errors: EINVAL (unknown pc, not a GLOBAL memory site, k too large), ESTATE, ENOSPC. */
 int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
 
+/* Top-K per-PC matrices: from the tables of the folds so far, rank the
+ * GLOBAL memory sites by distinct 32 B sectors per warp access (mem[s][2] / mem[s][0], compared
+ * exactly; ties: more warp accesses first, then the lower site index; sites never accessed are not
+ * ranked), then sassi_reset the context and keep the per-PC matrices of the first min(k, ranked)
+ * sites (sassi_select_memdiv_pcs) for the next pass over the same records. pcs_out (HOST, k
+ * entries) receives their pcs in rank order, *n_out their number. Synchronises `stream`.
+ * Errors: EINVAL (k > SASSI_MAX_PC_MATRICES, null pointer), ESTATE (peer tables attached). */
+int sassi_select_memdiv_topk(struct sassi_ctx* ctx, uint32_t k, uint32_t* pcs_out, uint32_t* n_out,
+                             void* stream);
+
 /* Dynamic sites: Fig.4 l.21-23 (L239) "Find the instruction's counters in a
  * hash table based on its address. Create a new entry if one does not exist." With this enabled,
  * every record whose pc is NOT registered (still counted in diag n_unknown_pc; it carries no rows)

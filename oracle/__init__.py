@@ -118,6 +118,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_select_pcs.restype = None
         L.oracle_dynamic_pcs.argtypes = [vp, u32, vp, u64, vp, u64, vp]
         L.oracle_dynamic_pcs.restype = u64
+        L.oracle_memdiv_topk.argtypes = [vp, u32, u32, vp, u32, vp]
+        L.oracle_memdiv_topk.restype = u32
         L.oracle_locate_injection.argtypes = [vp, u32, vp, u64, vp, u64, u64, u32, u32, vp]
         L.oracle_locate_injection.restype = ctypes.c_int
         _lib = L
@@ -178,6 +180,15 @@ def sample(counts: np.ndarray, k: int, seed: int) -> np.ndarray:
     if rc != 0:
         raise ValueError("oracle_sample: no eligible dynamic instruction to sample")
     return out
+
+
+def memdiv_topk(table: np.ndarray, sites, n_warps: int, k: int) -> list:
+    """Site indices of the k most divergent GLOBAL memory sites of a table (reading R26)."""
+    sites = np.ascontiguousarray(sites, dtype=SITE_DTYPE)
+    out = np.zeros(max(k, 1), np.uint32)
+    n = lib().oracle_memdiv_topk(sites.ctypes.data, len(sites), n_warps,
+                                 np.ascontiguousarray(table).ctypes.data, k, out.ctypes.data)
+    return [int(x) for x in out[:n]]
 
 
 def splitmix64(x: int) -> int:

@@ -49,6 +49,7 @@ SIGNATURES = {
     "sassi_ctx_destroy": (None, [_vp]),
     "sassi_attach_handler": (_i, [_vp, _u32]),
     "sassi_select_memdiv_pcs": (_i, [_vp, _vp, _u32]),
+    "sassi_select_memdiv_topk": (_i, [_vp, _u32, _vp, ctypes.POINTER(_u32), _vp]),
     "sassi_consume": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_consume_host": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_index_records": (_i, [_vp, _vp, _u64, _vp, _vp]),
@@ -173,6 +174,15 @@ def sassi_attach_handler(ctx: int, kind_mask: int) -> None:
 def sassi_select_memdiv_pcs(ctx: int, pcs) -> None:
     a = np.ascontiguousarray(pcs, dtype=np.uint32)
     _check(lib().sassi_select_memdiv_pcs(ctx, a.ctypes.data if a.size else None, a.size))
+
+
+def sassi_select_memdiv_topk(ctx: int, k: int, stream=None) -> np.ndarray:
+    """Rank GLOBAL memory sites by sectors per warp access in the tables so far, reset, and keep
+    the per-PC matrices of the top k for the next pass -> their pcs in rank order."""
+    out = np.zeros(max(k, 1), dtype=np.uint32)
+    n = _u32()
+    _check(lib().sassi_select_memdiv_topk(ctx, k, out.ctypes.data, ctypes.byref(n), _stream(stream)))
+    return out[:n.value]
 
 
 def sassi_consume(ctx: int, rec: dict, n=None, stream=None) -> None:
@@ -315,6 +325,10 @@ class Context:
     def select_memdiv_pcs(self, pcs) -> None:
         """Keep per-PC memory-divergence matrices (pcmat) for up to 4 GLOBAL memory sites."""
         sassi_select_memdiv_pcs(self.handle, pcs)
+
+    def select_memdiv_topk(self, k: int, stream=None) -> np.ndarray:
+        """Top-k most divergent GLOBAL pcs of the folds so far; resets and keeps their matrices."""
+        return sassi_select_memdiv_topk(self.handle, k, stream)
 
     def read_tables(self, stream=None) -> np.ndarray:
         return sassi_read_tables(self.handle, self.layout["total"], stream)

@@ -475,3 +475,27 @@ def test_select_memdiv_pcs_errors():
     ctx.select_memdiv_pcs([0x20])
     ctx.select_memdiv_pcs([])
     ctx.close()
+
+
+@pytest.mark.parametrize("k", [1, 4])
+def test_memdiv_topk_two_pass(k):
+    """sassi_select_memdiv_topk: pass 1 folds c2 (10^7 records), the k most
+    divergent GLOBAL pcs by sectors per warp access are picked (== the oracle's ranking of the
+    oracle's table, reading R26), the context is reset, and pass 2 keeps their matrices: every
+    table equals the oracle run with that selection."""
+    P, mask, d = _gen("c2", limit=2_000_000)
+    h = gen.to_host(d)
+    S, W = len(h["sites"]), P.total_warps
+    o1 = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+    want = oracle.memdiv_topk(o1, h["sites"], W, k)
+    ctx = sassi.Context(h["sites"], W, mask)
+    ctx.consume(d)
+    got = ctx.select_memdiv_topk(k)
+    assert [int(x) for x in got] == [int(h["sites"]["pc"][i]) for i in want]
+    assert np.array_equal(ctx.read_tables(), oracle.table_init(S, W, mask, pcs=want))  # reset
+    ctx.consume(d)
+    t = ctx.read_tables()
+    ctx.close()
+    o2 = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"], pcs=want)
+    assert diff_tables(t, o2, S, W) is None
+    assert oracle.sections(t, S, W)["pcmat"][:k].sum() > 0
