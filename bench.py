@@ -506,6 +506,9 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
     if not args.no_e2e:  # every rank at once on its own shard; the merge is inside the step at N > 1
         e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev, comm=comm, world=world,
                           launched=launched)
+        if extras and mask & 2:  # the same with the non-GLOBAL address rows split off
+            e2e["global_rows_only"] = measure_e2e(rec, P, mask, min(n, 1 << 24), dev, comm=comm,
+                                                  world=world, launched=launched, global_rows=True)
 
     cpu = slow = online = inj = None
     if extras and not args.no_cpu_baseline and rank == 0 and world == 1:
@@ -701,22 +704,31 @@ def measure_online_trace(dev, slow=None):
     return out
 
 
-def measure_e2e(rec, P, mask, n_e2e, dev, comm=None, world=1, launched=False):
+def measure_e2e(rec, P, mask, n_e2e, dev, comm=None, world=1, launched=False, global_rows=False):
     """records/s through sassi_consume_host: pinned host buffers of the first n_e2e records, the
     H2D copies (double-buffered inside the library) and the table read-back inside the timing.
     At N > 1 every rank does the same on its own shard at the same time (after a barrier), the
-    step includes the NCCL merge, and the time is the maximum over ranks."""
+    step includes the NCCL merge, and the time is the maximum over ranks. global_rows: the producer
+    split off the address rows of non-GLOBAL memory sites (SASSI_ADDR_ROWS_GLOBAL), which no
+    handler reads, so they never cross PCIe."""
     import torch
     import torch.distributed as dist
-    from paper_conf_isca_stephensonhlejn15_b200 import sassi
+    from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi
     n_e2e = (n_e2e // 256) * 256
     cb = rec["chunk_base"][: n_e2e // 256 + 1]
     tail = cb[-1].cpu().numpy().view(np.uint64)
     na, nv = int(tail[0]), int(tail[1])
-    h = dict(hdr=rec["hdr"][:n_e2e].cpu().pin_memory(), addr=rec["addr"][:na].cpu().pin_memory(),
-             val=rec["val"][:nv].cpu().pin_memory(), chunk_base=cb.cpu().pin_memory(), n=n_e2e,
-             n_addr_rows=na, n_val_rows=nv)
+    src = dict(rec, hdr=rec["hdr"][:n_e2e], addr=rec["addr"][:na], val=rec["val"][:nv],
+               chunk_base=cb, n=n_e2e, n_addr_rows=na, n_val_rows=nv)
+    if global_rows:  # producer-side split (input preparation, untimed)
+        src = gen.split_global_rows(src)
+        na = src["n_addr_rows"]
+    h = dict(hdr=src["hdr"].cpu().pin_memory(), addr=src["addr"].cpu().pin_memory(),
+             val=src["val"].cpu().pin_memory(), chunk_base=src["chunk_base"].cpu().pin_memory(),
+             n=n_e2e, n_addr_rows=na, n_val_rows=nv)
     ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=dev.index)
+    if global_rows:
+        ctx.set_addr_rows(sassi.SASSI_ADDR_ROWS_GLOBAL)
     stream = torch.cuda.current_stream(dev)
     out = np.zeros(ctx.layout["total"], np.uint64)
     cm = None
@@ -757,9 +769,10 @@ def measure_e2e(rec, P, mask, n_e2e, dev, comm=None, world=1, launched=False):
     return {"value": world * reps * n_e2e / el, "unit": "records/s", "h2d_bytes_per_step": world * h2d,
             "d2h_bytes_per_step": world * 8 * ctx.layout["total"], "records_per_step": world * n_e2e,
             "h2d_gbs": world * reps * h2d / el / 1e9,
-            "note": "pinned host buffers, first %d records of each rank's shard; wall clock around "
-                    "consume_host%s + read_tables (which synchronise), max over ranks" % (
-                        n_e2e, " + merge" if cm is not None else "")}
+            "note": "pinned host buffers, first %d records of each rank's shard%s; wall clock "
+                    "around consume_host%s + read_tables (which synchronise), max over ranks" % (
+                        n_e2e, ", address rows of GLOBAL memory sites only (SASSI_ADDR_ROWS_GLOBAL)"
+                        if global_rows else "", " + merge" if cm is not None else "")}
 
 
 if __name__ == "__main__":

@@ -212,6 +212,17 @@ int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
  * Errors: EINVAL (unknown pc, not a GLOBAL memory site, k too large), ESTATE, ENOSPC. */
 int sassi_select_memdiv_pcs(struct sassi_ctx* ctx, const uint32_t* pcs, uint32_t k);
 
+/* Address-row layout of the record streams this context consumes. SASSI_ADDR_ROWS_ALL (default,
+ * SRF1 as above): an addr row for every record at a SASSI_F_MEM site, any domain.
+ * SASSI_ADDR_ROWS_GLOBAL: the producer writes the rows of GLOBAL memory sites to the addr stream
+ * and the others (shared, local, ... memory, which no handler reads: memdiv counts GLOBAL only,
+ * L363 l.7) to a stream of their own that is not passed here; chunk_base's addr_row counts the
+ * GLOBAL rows only (sassi_index_records follows this setting). sassi_consume_host then copies only
+ * those rows over PCIe. Only before the first consume or right after sassi_reset.
+ * Errors: EINVAL, ESTATE. */
+enum { SASSI_ADDR_ROWS_ALL = 0u, SASSI_ADDR_ROWS_GLOBAL = 1u };
+int sassi_set_addr_rows(struct sassi_ctx* ctx, uint32_t which);
+
 /* Top-K per-PC matrices: from the tables of the folds so far, rank the
  * GLOBAL memory sites by distinct 32 B sectors per warp access (mem[s][2] / mem[s][0], compared
  * exactly; ties: more warp accesses first, then the lower site index; sites never accessed are not

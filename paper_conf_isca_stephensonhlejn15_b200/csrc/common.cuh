@@ -89,6 +89,8 @@ struct ConsumeParams {
   unsigned long long* peers[kMaxPeers];  // fused merge: peers' table images (same layout) ...
   uint32_t n_peers;                 // ... that every flush atomic also goes to
   uint32_t gmode;                   // 1: global mode (site table beyond shared memory)
+  uint32_t arow_bit;                // info bit of records with an address row in the stream:
+                                    // I_ADDR_ROW (every MEM site), I_MEMDIV (GLOBAL-only rows)
 };
 
 // home slot of an unregistered pc in the dynamic table (Fibonacci hashing: dense pcs spread)
@@ -141,6 +143,7 @@ struct sassi_ctx {
   uint32_t hmul = 1, hshr = 4;      // pc_slot parameters of the table on the device
   uint32_t nb = 0, nm = 0, nv = 0, nvd = 0, pw = 0, priv = 1;
   uint32_t gmode = 0;               // site table beyond shared memory: hash / state / counters global
+  uint32_t addr_global_only = 0;    // address row streams carry GLOBAL memory sites' rows only
   uint32_t pw_base = 0;             // private words of the branch / memdiv / value counters
   std::vector<uint32_t> mix_cat;    // per site: Fig.3 category bits (bit c = dynamic_instr_counts[c])
   uint32_t pcsel[4] = {0, 0, 0, 0}; // per-PC memdiv matrices: site index + 1 (0 = unused)

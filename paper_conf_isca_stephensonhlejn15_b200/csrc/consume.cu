@@ -550,7 +550,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       // ---- row indices of this batch (rows follow their records); only handlers that read
       // payload rows need them, header-only handler sets skip the bookkeeping ----
       constexpr bool kRows = (H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) != 0;
-      const uint32_t ma = kRows ? __ballot_sync(FULL, info & I_ADDR_ROW) : 0u;
+      const uint32_t ma = kRows ? __ballot_sync(FULL, info & p.arow_bit) : 0u;
       const uint32_t nd = (info >> I_NDST_SHIFT) & 7u;
       uint32_t vpre = 0, vtot = 0;
       if (kRows) {

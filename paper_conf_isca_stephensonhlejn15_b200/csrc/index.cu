@@ -10,7 +10,7 @@ namespace {
 __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restrict__ hdr, uint64_t n,
                                                            const uint4* __restrict__ hash,
                                                            uint32_t cap, uint32_t hmul, uint32_t hshr,
-                                                           uint64_t* na, uint64_t* nv) {
+                                                           uint32_t arow_bit, uint64_t* na, uint64_t* nv) {
   const uint64_t c = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t nch = (n + SASSI_CHUNK - 1) / SASSI_CHUNK;
@@ -26,7 +26,7 @@ __global__ void __launch_bounds__(256) chunk_counts_kernel(const uint4* __restri
       const uint32_t key = e.x;
       if (key == pc) {
         const uint32_t inf = e.y;
-        a += (inf & I_ADDR_ROW) ? 1u : 0u;
+        a += (inf & arow_bit) ? 1u : 0u;  // I_ADDR_ROW, or I_MEMDIV for GLOBAL-only address rows
         v += (inf >> I_NDST_SHIFT) & 7u;
         break;
       }
@@ -60,7 +60,8 @@ int launch_index(sassi_ctx* c, const sassi_hdr* hdr, uint64_t n, sassi_chunk_bas
   uint64_t *na = buf, *nv = buf + nch, *Pa = nv + nch, *Pv = Pa + nch + 1, *scratch = Pv + nch + 1;
   if (nch) {
     chunk_counts_kernel<<<(unsigned)((nch * 32 + 255) / 256), 256, 0, s>>>(
-        reinterpret_cast<const uint4*>(hdr), n, c->d_hash, c->cap, c->hmul, c->hshr, na, nv);
+        reinterpret_cast<const uint4*>(hdr), n, c->d_hash, c->cap, c->hmul, c->hshr,
+        c->addr_global_only ? I_MEMDIV : I_ADDR_ROW, na, nv);
     SASSI_CUDA(cudaGetLastError());
   }
   int rc = scan_u64(na, nch, Pa, scratch, s);

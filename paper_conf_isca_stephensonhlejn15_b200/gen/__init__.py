@@ -256,6 +256,45 @@ def to_host(rec: dict) -> dict:
     return out
 
 
+def split_global_rows(rec: dict) -> dict:
+    """The producer-side split of SASSI_ADDR_ROWS_GLOBAL (include/sassi.h): keep only the address
+    rows of GLOBAL memory sites (the rows of shared / local memory sites go to a stream of their own
+    that the fold never reads) and rebuild chunk_base's addr_row column over the kept rows. Works on
+    device (torch) and host (numpy) streams; input preparation only, no handler arithmetic."""
+    sites = rec["sites"]
+    order = np.argsort(sites["pc"].astype(np.int64))
+    spc = sites["pc"].astype(np.int64)[order]
+    mem = (sites["flags"][order].astype(np.int64) & F_MEM) != 0
+    glob = mem & (sites["domain"][order] == D_GLOBAL)
+    n = rec["n"]
+    if isinstance(rec["hdr"], np.ndarray):
+        pc = rec["hdr"]["pc"].astype(np.int64)[:n]
+        idx = np.minimum(np.searchsorted(spc, pc), max(len(spc) - 1, 0))
+        hit = (spc[idx] == pc) if len(spc) else np.zeros(n, bool)
+        has_row, is_g = hit & mem[idx], hit & glob[idx]
+        keep = is_g[has_row]
+        cum = np.concatenate([[0], np.cumsum(is_g)]).astype(np.uint64)
+        cb = rec["chunk_base"].copy()
+        cb[:, 0] = cum[np.minimum(np.arange(len(cb)) * CHUNK, n)]
+        addr = rec["addr"][keep]
+    else:
+        import torch
+        dev = rec["hdr"].device
+        tspc = torch.from_numpy(spc).to(dev)
+        pc = rec["hdr"][:n, 0].to(torch.int64) & 0xFFFFFFFF
+        idx = torch.clamp(torch.searchsorted(tspc, pc), max=max(len(spc) - 1, 0))
+        hit = tspc[idx] == pc
+        has_row = hit & torch.from_numpy(mem).to(dev)[idx]
+        is_g = hit & torch.from_numpy(glob).to(dev)[idx]
+        keep = is_g[has_row]
+        cum = torch.cat([torch.zeros(1, dtype=torch.int64, device=dev), torch.cumsum(is_g.to(torch.int64), 0)])
+        cb = rec["chunk_base"].clone()
+        pos = torch.clamp(torch.arange(cb.shape[0], device=dev) * CHUNK, max=n)
+        cb[:, 0] = cum[pos]
+        addr = rec["addr"][: rec["n_addr_rows"]][keep]
+    return dict(rec, addr=addr, chunk_base=cb, n_addr_rows=int(keep.sum()))
+
+
 def stream_bytes(rec: dict, handler_mask: int) -> dict:
     """Algorithmic bytes the fold must read for this stream and handler mask:
     16 B per header + 256 B per addr row of a GLOBAL memory site when MEMDIV is attached +

@@ -26,6 +26,7 @@ SASSI_ENOSPC, SASSI_ESTATE, SASSI_EMISMATCH, SASSI_EFORMAT = -4, -5, -6, -7
 SASSI_H_BRANCH, SASSI_H_MEMDIV, SASSI_H_VALUE, SASSI_H_INSTCOUNT, SASSI_H_ALL = 1, 2, 4, 8, 15
 SASSI_H_INSTMIX, SASSI_H_EVERY = 16, 31
 SASSI_CHUNK = 256
+SASSI_ADDR_ROWS_ALL, SASSI_ADDR_ROWS_GLOBAL = 0, 1
 SASSI_IK_VECADD, SASSI_IK_BFS, SASSI_IK_SGEMM, SASSI_IK_STENCIL = 0, 1, 2, 3
 SASSI_IK_NONE, SASSI_IK_TRACE, SASSI_IK_NULL_ABI, SASSI_IK_SMEM = 0, 64, 128, 1024
 
@@ -50,6 +51,7 @@ SIGNATURES = {
     "sassi_attach_handler": (_i, [_vp, _u32]),
     "sassi_select_memdiv_pcs": (_i, [_vp, _vp, _u32]),
     "sassi_select_memdiv_topk": (_i, [_vp, _u32, _vp, ctypes.POINTER(_u32), _vp]),
+    "sassi_set_addr_rows": (_i, [_vp, _u32]),
     "sassi_consume": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_consume_host": (_i, [_vp, ctypes.POINTER(SassiRecords), _u64, _vp]),
     "sassi_index_records": (_i, [_vp, _vp, _u64, _vp, _vp]),
@@ -174,6 +176,10 @@ def sassi_attach_handler(ctx: int, kind_mask: int) -> None:
 def sassi_select_memdiv_pcs(ctx: int, pcs) -> None:
     a = np.ascontiguousarray(pcs, dtype=np.uint32)
     _check(lib().sassi_select_memdiv_pcs(ctx, a.ctypes.data if a.size else None, a.size))
+
+
+def sassi_set_addr_rows(ctx: int, which: int) -> None:
+    _check(lib().sassi_set_addr_rows(ctx, which))
 
 
 def sassi_select_memdiv_topk(ctx: int, k: int, stream=None) -> np.ndarray:
@@ -325,6 +331,10 @@ class Context:
     def select_memdiv_pcs(self, pcs) -> None:
         """Keep per-PC memory-divergence matrices (pcmat) for up to 4 GLOBAL memory sites."""
         sassi_select_memdiv_pcs(self.handle, pcs)
+
+    def set_addr_rows(self, which: int) -> None:
+        """SASSI_ADDR_ROWS_GLOBAL: the streams carry the address rows of GLOBAL memory sites only."""
+        sassi_set_addr_rows(self.handle, which)
 
     def select_memdiv_topk(self, k: int, stream=None) -> np.ndarray:
         """Top-k most divergent GLOBAL pcs of the folds so far; resets and keeps their matrices."""

@@ -171,3 +171,24 @@ def test_c2_shape():
     assert 0.04 < int(sec["br"][:, 4].sum()) / nbr < 0.20
     assert 0.2 < r["n_addr_rows"] / n < 0.4
     assert 0.6 < r["n_val_rows"] / n < 0.9
+
+
+def test_split_global_rows_host():
+    """SASSI_ADDR_ROWS_GLOBAL input preparation: the kept rows are exactly the rows of the records
+    at GLOBAL memory sites, in record order, and chunk_base's addr_row counts them."""
+    P, _, _, _ = gen.preset("c3")
+    r = gen.generate_host(P, 5000, 0, 4)
+    g = gen.split_global_rows(r)
+    site = {int(x["pc"]): x for x in r["sites"]}
+    rows, kept, cnt = 0, [], [0]
+    for i, h in enumerate(r["hdr"]):
+        st = site.get(int(h["pc"]))
+        if st is not None and int(st["flags"]) & gen.F_MEM:
+            if int(st["domain"]) == gen.D_GLOBAL:
+                kept.append(rows)
+            rows += 1
+        cnt.append(len(kept))
+    assert g["n_addr_rows"] == len(kept) < r["n_addr_rows"]
+    assert np.array_equal(g["addr"], r["addr"][kept])
+    assert [int(x) for x in g["chunk_base"][:, 0]] == [cnt[min(256 * c, r["n"])] for c in range(len(g["chunk_base"]))]
+    assert np.array_equal(g["chunk_base"][:, 1], r["chunk_base"][:, 1])

@@ -499,3 +499,45 @@ def test_memdiv_topk_two_pass(k):
     o2 = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"], pcs=want)
     assert diff_tables(t, o2, S, W) is None
     assert oracle.sections(t, S, W)["pcmat"][:k].sum() > 0
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_global_only_address_rows_random(seed):
+    """SASSI_ADDR_ROWS_GLOBAL: the same records with only the GLOBAL sites' address rows (the
+    shared-memory rows split off by the producer) fold to the oracle's tables of the full stream;
+    sassi_index_records follows the layout."""
+    s, W, hdr, addr, val = random_trace(6100 + seed, n=20000)
+    o = oracle.run(s, W, sassi.SASSI_H_EVERY, hdr, addr, val)
+    full = to_device(s, hdr, addr, val)
+    d = gen.split_global_rows(dict(full, sites=s))
+    assert d["n_addr_rows"] < full["n_addr_rows"]
+    ctx = sassi.Context(s, W, sassi.SASSI_H_EVERY)
+    ctx.set_addr_rows(sassi.SASSI_ADDR_ROWS_GLOBAL)
+    cb = torch.zeros_like(d["chunk_base"])
+    sassi.sassi_index_records(ctx.handle, d["hdr"], d["n"], cb)
+    torch.cuda.synchronize()
+    assert torch.equal(cb, d["chunk_base"])
+    ctx.consume(d)
+    assert diff_tables(ctx.read_tables(), o, len(s), W) is None
+    ctx.close()
+
+
+def test_global_only_address_rows_c3_host_consume():
+    """c3 (2x10^6-record prefix, 12 % shared-memory records) from HOST buffers with the shared rows
+    split off: sassi_consume_host copies only the GLOBAL rows and the tables equal the oracle."""
+    P, mask, d = _gen("c3", limit=2_000_128)
+    h = gen.to_host(d)
+    g = gen.split_global_rows(h)
+    S, W = len(h["sites"]), P.total_warps
+    ctx = sassi.Context(h["sites"], W, mask)
+    ctx.set_addr_rows(sassi.SASSI_ADDR_ROWS_GLOBAL)
+    ctx.consume_host(dict(hdr=np.ascontiguousarray(g["hdr"]), addr=g["addr"], val=g["val"],
+                          chunk_base=g["chunk_base"], n=g["n"], n_addr_rows=g["n_addr_rows"],
+                          n_val_rows=g["n_val_rows"]))
+    t = ctx.read_tables()
+    with pytest.raises(sassi.SassiError):
+        ctx.set_addr_rows(sassi.SASSI_ADDR_ROWS_ALL)          # after a consume: ESTATE
+    ctx.close()
+    o = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+    assert diff_tables(t, o, S, W) is None
+    assert g["n_addr_rows"] < h["n_addr_rows"]
