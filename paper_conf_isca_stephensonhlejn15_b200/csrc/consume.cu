@@ -118,12 +118,16 @@ __device__ __forceinline__ void count_sorted(T v, uint32_t n, uint32_t lane, uin
 // are pairwise distinct (equal lines hash alike). The lanes then clear their words again.
 __device__ __forceinline__ bool lines_distinct(uint32_t line, bool in, uint32_t* bm, uint32_t mul) {
   const uint32_t h = (line * mul) >> (32 - SASSI_HASH_LG);
-  uint32_t* const w = bm + (h >> 5);
+  const uint32_t w = (uint32_t)__cvta_generic_to_shared(bm) + 4u * (h >> 5);
   const uint32_t bit = 1u << (h & 31u);
-  const uint32_t old = in ? atomicOr(w, bit) : 0u;
+  uint32_t old;
+  // predicated shared atomic / store (no branch around them)
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %1, 0; mov.u32 %0, 0; @q atom.shared.or.b32 %0, [%2], %3; }"
+               : "=r"(old) : "r"((uint32_t)in), "r"(w), "r"(bit) : "memory");
   const bool ok = !__any_sync(FULL, (old & bit) != 0u);
   __syncwarp();
-  if (in) *w = 0u;
+  asm volatile("{ .reg .pred q; setp.ne.u32 q, %0, 0; @q st.shared.u32 [%1], %2; }"
+               :: "r"((uint32_t)in), "r"(w), "r"(0u) : "memory");
   __syncwarp();
   return ok;
 }
