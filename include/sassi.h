@@ -199,7 +199,8 @@ void sassi_ctx_destroy(struct sassi_ctx* ctx);
  * the per-site counters in each SM's shared memory when they fit; a larger site table (thousands
  * of sites, up to SASSI_MAX_SITES) runs in "global mode": hash lookups from global memory and
  * per-record u64 atomics into the table image (the paper's own device-global tables),
- * same results, lower throughput. Errors: EINVAL, ESTATE, ENOSPC (the 32x32 matrices and the
+ * same results, lower throughput (the environment variable SASSI_FORCE_GLOBAL_MODE=1, read here,
+ * forces global mode for tests). Errors: EINVAL, ESTATE, ENOSPC (the 32x32 matrices and the
  * per-PC matrices alone exceed shared memory: not reachable with SASSI_MAX_PC_MATRICES). */
 int sassi_attach_handler(struct sassi_ctx* ctx, uint32_t kind_mask);
 

@@ -140,3 +140,24 @@ def test_one_site_too_many_is_enospc():
     with pytest.raises(sassi.SassiError) as e:
         sassi.sassi_ctx_create(0, _sites(65537, oracle.F_NUMERIC), 8)
     assert e.value.status == sassi.SASSI_ENOSPC
+
+
+@pytest.mark.parametrize("seed,n", [(1, 257), (2, 5000), (3, 20000)])
+@pytest.mark.parametrize("mask", [sassi.SASSI_H_ALL, sassi.SASSI_H_EVERY, sassi.SASSI_H_INSTMIX | 1])
+def test_forced_global_mode_random_traces(monkeypatch, seed, n, mask):
+    """Every handler path of global mode on the random edge-case traces (SASSI_FORCE_GLOBAL_MODE=1
+    puts small site tables through it), with per-PC matrices and dynamic pcs."""
+    from test_oracle import random_trace
+    monkeypatch.setenv("SASSI_FORCE_GLOBAL_MODE", "1")
+    s, W, hdr, addr, val = random_trace(8800 + seed, n=n)
+    glob = [i for i in range(len(s)) if (int(s[i]["flags"]) & oracle.F_MEM) and int(s[i]["domain"]) == 0]
+    ctx = sassi.Context(s, W, mask)
+    ctx.select_memdiv_pcs([int(s[i]["pc"]) for i in glob[:2]])
+    ctx.enable_dynamic_pcs(8)
+    ctx.consume(to_device(s, hdr, addr, val))
+    t = ctx.read_tables()
+    dyn, dropped = ctx.read_dynamic_pcs()
+    ctx.close()
+    assert diff_tables(t, oracle.run(s, W, mask, hdr, addr, val, pcs=glob[:2]), len(s), W) is None
+    odyn, odrop = oracle.dynamic_pcs(s, hdr)
+    assert dropped == odrop and [[int(e["pc"]), int(e["warp_execs"]), int(e["thread_execs"])] for e in dyn] == odyn.tolist()
