@@ -102,7 +102,9 @@ def lib() -> ctypes.CDLL:
             raise RuntimeError("libsassi.so not built (%s): run __graft_entry__.build()" % LIB_PATH)
         L = ctypes.CDLL(LIB_PATH)
         for name, (res, args) in SIGNATURES.items():
-            f = getattr(L, name)
+            f = getattr(L, name, None)
+            if f is None:  # an older build (SASSI_LIB A/B variants): calling it raises AttributeError
+                continue
             f.restype = res
             f.argtypes = args
         _lib = L
