@@ -309,6 +309,23 @@ int sassi_sample_sites(struct sassi_ctx* ctx, uint32_t k, uint64_t seed, sassi_i
 int sassi_sample_sites_device(struct sassi_ctx* ctx, uint32_t k, uint64_t seed,
                               sassi_inj_site* dev_out, uint32_t* dev_status, void* stream);
 
+/* An injection campaign over several kernel invocations (L629 "the static kernel name, dynamic
+ * kernel invocation ID, thread ID, dynamic instruction count"): one profile per invocation, each a
+ * context whose per-thread counts (SASSI_H_INSTCOUNT) were folded from that invocation, with the
+ * kernel and invocation ids its tuples carry. k draws uniform over all eligible dynamic
+ * thread-instructions of all profiles, with replacement (reading R29): draw j takes
+ * kk = floor(splitmix64(seed + j) * total / 2^64) over the profiles' totals in the given order, the
+ * profile holding kk, then thread and dynamic index within it as sassi_sample_sites (one profile
+ * with ids 0, 0 gives exactly sassi_sample_sites' tuples). All contexts on one device; HOST
+ * profiles[n] and out[k]; synchronises `stream` once. Errors: EINVAL (null, duplicate context,
+ * several devices), ESTATE (a profile without warps, or nothing to sample). */
+typedef struct sassi_profile {
+  struct sassi_ctx* ctx;
+  uint32_t kernel, invocation;
+} sassi_profile;
+int sassi_sample_sites_multi(const sassi_profile* profiles, uint32_t n, uint32_t k, uint64_t seed,
+                             sassi_inj_site* host_out, void* stream);
+
 /* Multi-GPU: merge the tables of all ranks of `nccl_comm` (ncclComm_t) in place with one
  * ncclAllReduce(sum, uint64) over a packed image (AND masks carried as byte-expanded bits); with
  * dynamic pcs enabled, also an ncclAllGather of every rank's dynamic table, which each rank

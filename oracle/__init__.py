@@ -112,6 +112,8 @@ def lib() -> ctypes.CDLL:
         L.oracle_merge.restype = None
         L.oracle_sample.argtypes = [vp, u64, u32, u64, vp]
         L.oracle_sample.restype = ctypes.c_int
+        L.oracle_sample_multi.argtypes = [vp, vp, vp, vp, u32, u32, u64, vp]
+        L.oracle_sample_multi.restype = ctypes.c_int
         L.oracle_splitmix64.argtypes = [u64]
         L.oracle_splitmix64.restype = u64
         L.oracle_select_pcs.argtypes = [u32, u32, vp, u32, vp]
@@ -189,6 +191,20 @@ def memdiv_topk(table: np.ndarray, sites, n_warps: int, k: int) -> list:
     n = lib().oracle_memdiv_topk(sites.ctypes.data, len(sites), n_warps,
                                  np.ascontiguousarray(table).ctypes.data, k, out.ctypes.data)
     return [int(x) for x in out[:n]]
+
+
+def sample_multi(profiles, k: int, seed: int) -> np.ndarray:
+    """Draws over several kernel invocations: profiles = [(counts, kernel, invocation), ...]."""
+    counts = np.ascontiguousarray(np.concatenate([np.asarray(c, np.uint64) for c, _, _ in profiles]))
+    nt = np.array([len(c) for c, _, _ in profiles], np.uint64)
+    ke = np.array([kk for _, kk, _ in profiles], np.uint32)
+    iv = np.array([ii for _, _, ii in profiles], np.uint32)
+    out = np.zeros(k, dtype=INJ_DTYPE)
+    rc = lib().oracle_sample_multi(counts.ctypes.data, nt.ctypes.data, ke.ctypes.data, iv.ctypes.data,
+                                   len(profiles), k, seed & (2**64 - 1), out.ctypes.data)
+    if rc != 0:
+        raise ValueError("oracle_sample_multi: no eligible dynamic instruction to sample")
+    return out
 
 
 def splitmix64(x: int) -> int:

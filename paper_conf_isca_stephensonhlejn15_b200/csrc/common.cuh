@@ -206,6 +206,8 @@ int launch_sample(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* host_
                   cudaStream_t s);
 int launch_sample_device(sassi_ctx* c, uint32_t k, uint64_t seed, sassi_inj_site* dev_out,
                          uint32_t* dev_status, cudaStream_t s);
+int launch_sample_multi(sassi_ctx* const* ctxs, const uint32_t* kernel, const uint32_t* invocation,
+                        uint32_t n, uint32_t k, uint64_t seed, sassi_inj_site* host_out, cudaStream_t s);
 int launch_merge(sassi_ctx* c, void* comm, cudaStream_t s);
 int launch_merge_local(sassi_ctx* const* ctxs, uint32_t n, cudaStream_t s);
 int consume_smem_bytes(const sassi_ctx* c, size_t* bytes);

@@ -60,6 +60,7 @@ SIGNATURES = {
     "sassi_tables_device": (_i, [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_u64)]),
     "sassi_sample_sites": (_i, [_vp, _u32, _u64, _vp, _vp]),
     "sassi_sample_sites_device": (_i, [_vp, _u32, _u64, _vp, _vp, _vp]),
+    "sassi_sample_sites_multi": (_i, [_vp, _u32, _u32, _u64, _vp, _vp]),
     "sassi_merge": (_i, [_vp, _vp, _vp]),
     "sassi_merge_local": (_i, [_vp, _u32, _vp]),
     "sassi_nccl_get_unique_id": (_i, [_vp]),
@@ -238,6 +239,20 @@ def sassi_sample_sites_device(ctx: int, k: int, seed: int, dev_out: int, dev_sta
     dev_status (1 = nothing to sample)."""
     _check(lib().sassi_sample_sites_device(ctx, k, seed & (2**64 - 1), dev_out or None, dev_status,
                                            _stream(stream)))
+
+
+class SassiProfile(ctypes.Structure):
+    _fields_ = [("ctx", _vp), ("kernel", _u32), ("invocation", _u32)]
+
+
+def sassi_sample_sites_multi(profiles, k: int, seed: int, stream=None) -> np.ndarray:
+    """profiles = [(Context or handle, kernel id, invocation id), ...] -> k tuples (INJ_DTYPE)."""
+    arr = (SassiProfile * len(profiles))(*[SassiProfile(getattr(c, "handle", c), kk, ii)
+                                           for c, kk, ii in profiles])
+    out = np.zeros(k, dtype=INJ_DTYPE)
+    _check(lib().sassi_sample_sites_multi(arr, len(profiles), k, seed & (2**64 - 1),
+                                          out.ctypes.data if k else None, _stream(stream)))
+    return out
 
 
 def sassi_merge(ctx: int, comm: int, stream=None) -> None:

@@ -129,3 +129,42 @@ def test_injection_beyond_the_profile_is_not_reached():
     assert outs["outcome"][0] == sassi.SASSI_INJ_NOT_REACHED and outs["site"][0] == 0xFFFFFFFF
     assert outs["outcome"][1] != sassi.SASSI_INJ_NOT_REACHED
     ik.close()
+
+
+def test_campaign_across_kernels_and_invocations():
+    """§8.1 (L627, L629): one campaign over several kernel invocations — vecadd, stencil and two
+    invocations of BFS (different graphs) — drawn uniformly over all their eligible dynamic
+    instructions (sassi_sample_sites_multi == the oracle's draws over the concatenated profiles);
+    each tuple goes to its kernel invocation and hits what the oracle locates in that trace."""
+    kernels = [("vecadd", 12800, 20150613, 0, 0), ("stencil", 64, 20150613, 1, 0),
+               ("bfs", 4096, 20150613, 2, 0), ("bfs", 4096, 77, 2, 1)]
+    iks, ctxs, profiles, oprof, traces = [], [], [], [], []
+    for name, size, seed, kid, inv in kernels:
+        ik = sassi.InstrumentedKernel(name, size, seed=seed)
+        ctx = ik.context(sassi.SASSI_H_INSTCOUNT)
+        ik.run(sassi.SASSI_H_INSTCOUNT, ctx)
+        profiles.append((ctx, kid, inv))
+        oprof.append((ctx.sections()["counts"], kid, inv))
+        tctx = ik.context(sassi.SASSI_H_INSTCOUNT)
+        traces.append(gen.to_host(ik.trace(tctx)))
+        tctx.close()
+        iks.append(ik)
+        ctxs.append(ctx)
+    sites = sassi.sassi_sample_sites_multi(profiles, 400, 2024)
+    assert np.array_equal(sites, oracle.sample_multi(oprof, 400, 2024))
+    assert len(set(zip(sites["kernel"].tolist(), sites["invocation"].tolist()))) == 4
+    # one profile with ids 0 / 0 is sassi_sample_sites
+    assert np.array_equal(sassi.sassi_sample_sites_multi([(ctxs[0], 0, 0)], 50, 3), ctxs[0].sample(50, 3))
+    for i, (name, size, seed, kid, inv) in enumerate(kernels):
+        mine = sites[(sites["kernel"] == kid) & (sites["invocation"] == inv)]
+        outs = iks[i].inject(mine)
+        h = traces[i]
+        for st, o in zip(mine, outs):
+            loc = oracle.locate_injection(h["sites"], h["hdr"], h["val"], int(st["thread"]),
+                                          int(st["dyn_index"]), int(st["reg_seed"]), int(st["bit_seed"]))
+            assert loc is not None and int(o["site"]) == loc["site"] and int(o["bit"]) == loc["bit"]
+            assert int(o["target"]) == TARGET_CODE[loc["target"]]
+    for c in ctxs:
+        c.close()
+    for ik in iks:
+        ik.close()

@@ -541,3 +541,24 @@ def test_global_only_address_rows_c3_host_consume():
     o = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
     assert diff_tables(t, o, S, W) is None
     assert g["n_addr_rows"] < h["n_addr_rows"]
+
+
+def test_sample_sites_multi_random_profiles():
+    """sassi_sample_sites_multi over five random-trace profiles of different warp counts equals the
+    oracle's draws over the concatenated counts; a profile with nothing counted contributes none."""
+    profs, oprofs, ctxs = [], [], []
+    for i, (n, w) in enumerate([(3000, 5), (500, 1), (7000, 40), (1, 3), (20000, 70)]):
+        s, W, hdr, addr, val = random_trace(9100 + i, n=n, n_warps=w)
+        ctx = sassi.Context(s, W, sassi.SASSI_H_INSTCOUNT)
+        ctx.consume(to_device(s, hdr, addr, val))
+        c = oracle.sections(oracle.run(s, W, sassi.SASSI_H_INSTCOUNT, hdr, addr, val), len(s), W)["counts"]
+        profs.append((ctx, 10 + i, i))
+        oprofs.append((c, 10 + i, i))
+        ctxs.append(ctx)
+    for k, seed in ((1, 0), (33, 5), (1000, 2**40 + 3)):
+        assert np.array_equal(sassi.sassi_sample_sites_multi(profs, k, seed), oracle.sample_multi(oprofs, k, seed))
+    with pytest.raises(sassi.SassiError) as e:
+        sassi.sassi_sample_sites_multi([profs[0], profs[0]], 4, 1)
+    assert e.value.status == sassi.SASSI_EINVAL
+    for c in ctxs:
+        c.close()
