@@ -678,21 +678,21 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
             const uint32_t Vj = __shfl_sync(FULL, vsel, j);
             const uint32_t slot = __shfl_sync(FULL, vslot, j) + (r - __shfl_sync(FULL, vpre, j));
             const uint32_t V = lane < nr ? Vj : 0u;
-            // lane folds row s0+lane: 8 chunks of 4 values, chunk order rotated by lane so the 8
-            // lanes of each shared-memory phase hit 8 different bank groups
+            // lane folds row s0+lane: 8 chunks of 4 values, chunk k ^ (lane & 7) at step k so the
+            // 8 lanes of each shared-memory phase hit 8 different bank groups
             const uint4* row = vbuf + 8 * lane;
             uint32_t va = FULL, vo = 0;
             if (__all_sync(FULL, V == FULL || V == 0)) {
 #pragma unroll
               for (uint32_t k = 0; k < 8; ++k) {
-                const uint4 x = row[(k + lane) & 7u];
+                const uint4 x = row[k ^ (lane & 7u)];
                 va &= x.x & x.y & x.z & x.w;
                 vo |= x.x | x.y | x.z | x.w;
               }
             } else {
 #pragma unroll
               for (uint32_t k = 0; k < 8; ++k) {
-                const uint32_t c = (k + lane) & 7u;
+                const uint32_t c = k ^ (lane & 7u);
                 const uint4 x = row[c];
                 const uint32_t vb = V >> (4 * c);
                 const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
