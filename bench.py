@@ -350,14 +350,21 @@ def run_c5(args, rank, world, local):
     dev = torch.device("cuda", local)
     P, limit, mask, desc = gen.preset("c5")
     stream = torch.cuda.current_stream(dev)
-    comm = nccl_comm(world, rank, local, dev) if world > 1 else None
+    # the N > 1 parts (merge, T_1, weak scaling) also run at N = 1 with SASSI_BENCH_SCALING_EXTRAS=1
+    # (a 1-rank communicator), so the multi-GPU code path is exercised on a one-GPU box
+    multi = world > 1 or os.environ.get("SASSI_BENCH_SCALING_EXTRAS") == "1"
+    comm = nccl_comm(world, rank, local, dev) if multi else None
+
+    def barrier():
+        if dist.is_initialized():
+            dist.barrier()
+
     draws = torch.empty(N_DRAWS * 32, dtype=torch.uint8, device=dev)
     status = torch.zeros(1, dtype=torch.int32, device=dev)
     with ClockSampler(local) as clk:
         job, consume_ms, n_total, alg_total = fold_c5_shards(args, range(rank, 8, world), P, mask,
                                                              dev, local)
-        if world > 1:
-            dist.barrier()
+        barrier()
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t0.record(stream)
         if comm is not None:
@@ -376,8 +383,8 @@ def run_c5(args, rank, world, local):
     job.close()
     t1_job = t1_shard_ms = None
     weak = None
-    if world > 1:
-        dist.barrier()
+    if multi:
+        barrier()
         if rank == 0:  # T_1: the same job on one GPU (all 8 shards, no merge)
             j1, ms1, _, _ = fold_c5_shards(args, range(8), P, mask, dev, local)
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -388,7 +395,7 @@ def run_c5(args, rank, world, local):
             t1_job = sum(ms1) / 1e3 + a.elapsed_time(b) / 1e3
             t1_shard_ms = ms1
             j1.close()
-        dist.barrier()
+        barrier()
         weak = run_weak(args, rank, world, local, "c3", extras=False, comm=comm,
                         steps=min(args.steps, 10))
     if comm is not None:
@@ -416,7 +423,7 @@ def run_c5(args, rank, world, local):
                              "frac": per_gpu_alg / t_shards / 1e9 / peak, "peak_source": peak_src,
                              "traffic": ncu_traffic("c5"), "consume_ms_per_shard": consume_ms},
                 "gpu_launches": launches, "clocks": clk.result()}
-        if world > 1:
+        if multi:
             line["strong_scaling"] = {
                 "t1_ms": 1e3 * t1_job, "tN_ms": 1e3 * t_job, "t1_consume_ms_per_shard": t1_shard_ms,
                 "note": "T_1 = rank 0 alone folding all 8 shards + sampling, same protocol, same run; "
@@ -440,7 +447,7 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
     dev = torch.device("cuda", local)
     steps = args.steps if steps is None else steps
     launched = dist.is_initialized()
-    merge_on = world > 1 or os.environ.get("SASSI_BENCH_FORCE_MERGE") == "1"
+    merge_on = world > 1 or comm is not None or os.environ.get("SASSI_BENCH_FORCE_MERGE") == "1"
     P, limit, desc = workload_program(workload, world)
     mask = gen.PRESETS[workload][2]
     per = P.total_warps // world
