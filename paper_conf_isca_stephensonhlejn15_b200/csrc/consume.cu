@@ -137,9 +137,9 @@ __device__ __forceinline__ bool lines_distinct(uint32_t line, bool in, uint32_t*
 //  - window path: every sector of G within the 32-sector (1 KB, 8-line) window that starts at the
 //    line holding the lowest sector (same high word): the window bitmap is OR-reduced across the
 //    warp (REDUX), s = its popcount, L = the popcount of its nibbles OR-folded (a nibble = a line).
-//  - otherwise, when all high words agree (gathers): if a hashed bitmap shows the lines of G to be
-//    pairwise distinct, s = L = |G| (lines_distinct, two rounds); else sort the 32-bit keys across
-//    the warp (bitonic) with the
+//  - otherwise (gathers): if a hashed bitmap shows the lines of G to be pairwise distinct,
+//    s = L = |G| (lines_distinct, two rounds); else, when all high words agree, sort the 32-bit
+//    keys across the warp (bitonic) with the
 //    lanes outside G padded to the maximum so they sort last, and count positions < n whose key
 //    differs from the previous one; lines come from the same sorted sectors (>> 2 keeps order).
 //  - rows whose sectors differ in the high word return false and go to memdiv_row64 (64-bit keys),
@@ -159,9 +159,10 @@ __device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t la
     *out_l = __popc((m | (m >> 1) | (m >> 2) | (m >> 3)) & 0x11111111u);
     return true;
   }
-  if (!__all_sync(FULL, same_hi)) return false;
   // scattered rows (gathers): if the lines of G are pairwise distinct, so are the sectors, and
-  // s = L = |G| with no sort; a hash collision or a repeated line falls through to the sort
+  // s = L = |G| with no sort; a hash collision or a repeated line falls through to the sort. The
+  // keys are the lines' low 30 bits: equal lines give equal keys, so distinct keys prove distinct
+  // lines whatever the high words (no uniformity check needed before the hash)
   if (SASSI_HASH_ROUNDS >= 1 && lines_distinct(slo >> 2, in, bm, 0x9E3779B1u)) {
     *out_s = *out_l = __popc(G);
     return true;
@@ -170,6 +171,7 @@ __device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t la
     *out_s = *out_l = __popc(G);
     return true;
   }
+  if (!__all_sync(FULL, same_hi)) return false;
   count_sorted(warp_sort<uint32_t>(in ? slo : FULL, lane), __popc(G), lane, out_s, out_l);
   return true;
 }
