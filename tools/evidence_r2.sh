@@ -20,3 +20,8 @@ for w in c3 c2 c4; do
   python tools/ncu_toplines.py /tmp/rep/consume_$w.ncu-rep consume.cu 40 > $O/toplines_$w.txt 2>&1
 done
 ls $O
+timeout 600 python tools/paper_report.py $O/paper_report.md > /dev/null 2>&1
+timeout 1200 python tools/fuzz_parity.py 300 11 > $O/fuzz_parity.txt 2>&1
+timeout 900 python tools/fuzz_inline.py > $O/fuzz_inline.txt 2>&1
+SASSI_BENCH_SCALING_EXTRAS=1 timeout 900 python bench.py --workload c5 --steps 10 > $O/bench_c5_scaling_extras.json 2>&1
+ls $O
