@@ -25,6 +25,9 @@
 #ifndef SASSI_HDR_DEPTH
 #define SASSI_HDR_DEPTH 3  // header batches in flight per warp (header-only handler sets)
 #endif
+#ifndef SASSI_ROW_GROUP
+#define SASSI_ROW_GROUP 3  // memdiv address rows loaded per group (measured: 3 beats 2, 4, 6)
+#endif
 #ifndef SASSI_HASH_LG
 #define SASSI_HASH_LG 11     // memdiv distinctness check: 2^11 bit buckets per warp (256 B)
 #endif
@@ -595,10 +598,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
           uint32_t my_s = 0, my_l = 0;  // results of this lane's own record
           uint32_t slow = 0;            // rows whose sectors differ in the high word
           do {
-            uint64_t a[4];
-            uint32_t g[4], jj[4];
+            uint64_t a[SASSI_ROW_GROUP];
+            uint32_t g[SASSI_ROW_GROUP], jj[SASSI_ROW_GROUP];
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {
+            for (int k = 0; k < SASSI_ROW_GROUP; ++k) {
               g[k] = 0;
               if (selm) {
                 const int j = __ffs(selm) - 1;
@@ -609,7 +612,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
               }
             }
 #pragma unroll
-            for (int k = 0; k < 4; ++k) {
+            for (int k = 0; k < SASSI_ROW_GROUP; ++k) {
               if (g[k]) {
                 uint32_t s, L;
                 if (memdiv_row32(a[k], g[k], lane, hbm, &s, &L)) {
