@@ -665,6 +665,15 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
           const uint32_t vsel = selv ? G : 0u;                // lanes written by this lane's record
           // its first value-state slot (global mode: 4 * site, the image's [S][4] words)
           const uint32_t vslot = gm ? 4u * e.w : (info >> I_VD0_SHIFT) & 0xFFFFu;
+          // the owner of every value row of the batch (lane ids in the warp's memdiv bitmap words,
+          // which are all zero between memdiv rows): each lane records itself for its nd rows
+          uint8_t* const owner = reinterpret_cast<uint8_t*>(hbm);
+          if (Ly::kMem) {
+#pragma unroll
+            for (uint32_t d = 0; d < 4; ++d)
+              if (d < nd) owner[vpre + d] = (uint8_t)lane;
+            __syncwarp();
+          }
           for (uint32_t s0 = 0; s0 < vtot; s0 += 32) {
             const uint32_t nr = min(vtot - s0, 32u);
             if (s0) {  // rows beyond the first 32: reuse the buffer once every lane is done with it
@@ -677,9 +686,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
             // value row, since a lane without rows shares vpre with its successor)
             const uint32_t r = s0 + lane;
             uint32_t j = 0;
+            if (Ly::kMem) {
+              j = owner[r & 127u];
+            } else {
 #pragma unroll
-            for (uint32_t step = 16; step; step >>= 1)
-              if (__shfl_sync(FULL, vpre, j + step) <= r) j += step;
+              for (uint32_t step = 16; step; step >>= 1)
+                if (__shfl_sync(FULL, vpre, j + step) <= r) j += step;
+            }
             const uint32_t Vj = __shfl_sync(FULL, vsel, j);
             const uint32_t slot = __shfl_sync(FULL, vslot, j) + (r - __shfl_sync(FULL, vpre, j));
             const uint32_t V = lane < nr ? Vj : 0u;
@@ -723,6 +736,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
             }
           }
           __syncwarp();
+          if (Ly::kMem) {  // the bitmap words back to zero for the next batch's memdiv rows
+            hbm[lane] = 0u;
+            __syncwarp();
+          }
         }
       }
     }
