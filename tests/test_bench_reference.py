@@ -94,6 +94,7 @@ def test_bench_multi_gpu_code_path_is_importable_and_documented():
     b = importlib.util.module_from_spec(spec)
     spec.loader.exec_module(b)
     src = open(os.path.join(ROOT, "bench.py")).read()
-    for key in ('"strong_scaling"', '"weak_scaling"', '"t1_ms"', "SASSI_BENCH_SCALING_EXTRAS", "self_launch"):
+    for key in ('"strong_scaling"', '"weak_scaling"', '"weak_scaling_c5"', '"t1_ms"', "SASSI_BENCH_SCALING_EXTRAS",
+                "self_launch"):
         assert key in src
     assert callable(b.run_c5) and callable(b.run_weak) and callable(b.self_launch)
