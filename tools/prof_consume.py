@@ -10,7 +10,8 @@ name = sys.argv[1] if len(sys.argv) > 1 else "c3"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 3
 mask = int(sys.argv[3]) if len(sys.argv) > 3 else gen.PRESETS[name][2]
 P, lim, _, _ = gen.preset(name)
-d = gen.generate_device(P, lim)
+# c5 (8 shards, ~680 GB) is profiled on one shard of 16,384 warps, as the bench folds it
+d = gen.generate_device(P, None, 0, 16384) if name == "c5" else gen.generate_device(P, lim)
 ctx = sassi.Context(d["sites"], P.total_warps, mask)
 for _ in range(reps):
     ctx.reset()
