@@ -708,15 +708,18 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
                 vo |= x.x | x.y | x.z | x.w;
               }
             } else {
+              // lanes outside V hold garbage: stand in the row's value at a lane of V for them
+              // (neutral for both AND and OR)
+              const uint32_t ref = V ? reinterpret_cast<const uint32_t*>(row)[__ffs(V) - 1] : 0u;
 #pragma unroll
               for (uint32_t k = 0; k < 8; ++k) {
                 const uint32_t c = k ^ (lane & 7u);
                 const uint4 x = row[c];
                 const uint32_t vb = V >> (4 * c);
-                const uint32_t m0 = 0u - (vb & 1u), m1 = 0u - ((vb >> 1) & 1u);
-                const uint32_t m2_ = 0u - ((vb >> 2) & 1u), m3 = 0u - ((vb >> 3) & 1u);
-                va &= (x.x | ~m0) & (x.y | ~m1) & (x.z | ~m2_) & (x.w | ~m3);
-                vo |= (x.x & m0) | (x.y & m1) | (x.z & m2_) | (x.w & m3);
+                const uint32_t x0 = (vb & 1u) ? x.x : ref, x1 = (vb & 2u) ? x.y : ref;
+                const uint32_t x2 = (vb & 4u) ? x.z : ref, x3 = (vb & 8u) ? x.w : ref;
+                va &= x0 & x1 & x2 & x3;
+                vo |= x0 | x1 | x2 | x3;
               }
             }
             if (V != 0 && !gm) {
