@@ -159,7 +159,8 @@ __device__ __forceinline__ bool memdiv_row32(uint64_t a, uint32_t G, uint32_t la
   if (__all_sync(FULL, same_hi && (!in || e < 32u))) {
     const uint32_t m = __reduce_or_sync(FULL, in ? (1u << e) : 0u);
     *out_s = __popc(m);
-    *out_l = __popc((m | (m >> 1) | (m >> 2) | (m >> 3)) & 0x11111111u);
+    const uint32_t t = m | (m >> 2);
+    *out_l = __popc((t | (t >> 1)) & 0x11111111u);
     return true;
   }
   // scattered rows (gathers): if the lines of G are pairwise distinct, so are the sectors, and
