@@ -50,6 +50,12 @@ def parse():
                     help="default: c3 at N = 1, c5 at N > 1")
     ap.add_argument("--selftest-dist", action="store_true",
                     help="launch / rendezvous / max-over-ranks plumbing only (gloo without a GPU)")
+    ap.add_argument("--merge", default="nccl", choices=["nccl", "p2p"],
+                    help="N > 1: sassi_merge over NCCL after the fold, or the fused fold + merge over "
+                         "peer memory (every rank's fold also updates the other ranks' images)")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="N > 1 ranks all on cuda:0 (gloo process group, --merge p2p; c2 / c3 / c4): "
+                         "the multi-rank code path on a one-GPU box, not a scaling measurement")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-slowdown", action="store_true")
@@ -477,7 +483,14 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
     alg_bytes, n_glob = algorithmic_bytes(rec, mask)
     ctx = sassi.Context(rec["sites"], P.total_warps, mask, device=local)
     own_comm = None
-    if merge_on and comm is None:
+    p2p = getattr(args, "merge", "nccl") == "p2p" and world > 1
+    if p2p:  # fused fold + merge: every rank's flush also updates the other ranks' images
+        handles = [None] * world
+        dist.all_gather_object(handles, ctx.ipc_table_handle())
+        for j in range(world):
+            if j != rank:
+                ctx.add_peer_table(handles[j])
+    elif merge_on and comm is None:
         comm = own_comm = nccl_comm(world, rank, local, dev)
     stream = torch.cuda.current_stream(dev)
     sample = bool(mask & 8)
@@ -487,11 +500,17 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
 
     def step(ev_c0=None, ev_c1=None):
         ctx.reset(stream)
+        if p2p:  # every image reset before any rank folds into it
+            torch.cuda.synchronize(dev)
+            dist.barrier()
         if ev_c0 is not None:
             ev_c0.record(stream)
         ctx.consume(rec, stream=stream)
         if ev_c1 is not None:
             ev_c1.record(stream)
+        if p2p:  # every rank's fold (and its flush into the peers) done before the draws
+            torch.cuda.synchronize(dev)
+            dist.barrier()
         if comm is not None:
             ctx.merge(comm, stream)
         if sample:
@@ -521,8 +540,11 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
         assert int(draw_status.item()) == 0, "sampling: no eligible dynamic instruction"
         host_draws = ctx.sample(N_DRAWS, 20150616, stream)
         assert draws.cpu().numpy().tobytes() == host_draws.tobytes(), "device draws differ"
-    ms = max_over_ranks(t_start.elapsed_time(t_end), dev)
+    ms = t_start.elapsed_time(t_end)
     consume_ms = [a.elapsed_time(b) for a, b in evs]
+    if p2p:  # the step is the fused fold + merge; the host barriers around it are not device time
+        ms = sum(consume_ms)
+    ms = max_over_ranks(ms, dev)
     sec = ms / 1e3
     value = world * n * steps / sec
     consume_avg_s = statistics.mean(consume_ms) / 1e3
@@ -531,7 +553,7 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
 
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
-    if not args.no_e2e:  # every rank at once on its own shard; the merge is inside the step at N > 1
+    if not args.no_e2e and not p2p:  # every rank at once on its own shard; the merge is inside the step at N > 1
         e2e = measure_e2e(rec, P, mask, min(n, 1 << 24), dev, comm=comm, world=world,
                           launched=launched)
         if extras and mask & 2:  # the same with the non-GLOBAL address rows split off
@@ -548,6 +570,9 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
         inj = measure_injection(dev)
     if own_comm is not None:
         sassi.sassi_nccl_comm_destroy(own_comm)
+    if p2p:  # (the p2p protocol's parity: tests/test_gpu_p2p.py)
+        ctx.clear_peer_tables()
+        dist.barrier()  # every handle to this image is closed before it is freed
     ctx.close()
     if rank != 0:
         return None
@@ -564,7 +589,9 @@ def run_weak(args, rank, world, local, workload, extras=True, comm=None, steps=N
                    "stored_bytes_per_gpu": stored, "algorithmic_bytes_per_gpu": alg_bytes,
                    "l2": "inputs (%.1f GB) exceed the 126 MB L2; no flush" % (stored / 1e9),
                    "parallelism": "dp%d (warp-id shards%s)" % (
-                       world, ", NCCL allreduce merge per step" if merge_on else "")},
+                       world, ", fused fold + merge over peer memory" if p2p else
+                       (", NCCL allreduce merge per step" if merge_on else "")),
+                   "shared_gpu": bool(getattr(args, "share_gpu", False))},
         "hbm_gbs": world * alg_bytes * steps / sec / 1e9,
         "hbm_frac_of_spec_8tbs": alg_bytes * steps / sec / 1e9 / SPEC_HBM_GBS,
         "roofline": {"bound": "hbm", "kernel": "consume_kernel<%d>" % mask,
@@ -600,9 +627,17 @@ def main():
         return
     import torch
     import torch.distributed as dist
+    if args.share_gpu:
+        if args.merge != "p2p" or args.workload == "c5":
+            sys.exit("bench.py: --share-gpu needs --merge p2p and c2 / c3 / c4 (NCCL refuses two ranks "
+                     "on one GPU; c5 shards do not fit twice)")
+        local = 0
     torch.cuda.set_device(local)
     if "RANK" in os.environ:  # under torchrun (any world size)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.share_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     try:
         if args.workload == "c5":
             run_c5(args, rank, world, local)

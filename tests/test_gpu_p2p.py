@@ -31,3 +31,25 @@ def test_fused_merge_two_processes(world):
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     for k in range(world):
         assert "p2p ok rank %d of %d" % (k, world) in r.stdout
+
+
+def test_bench_two_ranks_sharing_the_gpu_fused_merge():
+    """bench.py's N > 1 code path on a one-GPU box: `--gpus 2 --share-gpu --merge p2p` self-launches
+    two ranks (gloo), both on cuda:0, each folding its c2 warp shard into both table images; one
+    JSON line with n_gpus = 2 (the device-side draws are checked against the host-output draws
+    inside bench.py). Not a scaling measurement: the two ranks share one GPU."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import json
+    root = os.path.dirname(HERE)
+    cmd = [sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--share-gpu", "--merge", "p2p",
+           "--workload", "c2", "--steps", "3", "--warmup", "1", "--no-e2e", "--no-cpu-baseline",
+           "--no-slowdown", "--no-injection"]
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "WORLD_SIZE", "LOCAL_RANK")}
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, env=env, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    lines = [json.loads(l) for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = lines[0]
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["config"]["shared_gpu"] is True
+    assert "fused fold + merge over peer memory" in d["config"]["parallelism"]
