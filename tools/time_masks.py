@@ -8,8 +8,12 @@ from paper_conf_isca_stephensonhlejn15_b200 import gen, sassi  # noqa: E402
 
 name = sys.argv[1] if len(sys.argv) > 1 else "c3"
 masks = [int(m) for m in sys.argv[2].split(",")] if len(sys.argv) > 2 else [15, 4, 2, 1, 8, 9, 11, 13, 6]
-P, lim, _, _ = gen.preset(name)
-d = gen.generate_device(P, lim)
+if name == "c5s":  # one c5 warp shard (16,384 of the 131,072 warps, as bench.py folds them)
+    P, _, _, _ = gen.preset("c5")
+    d = gen.generate_device(P, None, 0, 16384)
+else:
+    P, lim, _, _ = gen.preset(name)
+    d = gen.generate_device(P, lim)
 s = torch.cuda.current_stream()
 for m in masks:
     ctx = sassi.Context(d["sites"], P.total_warps, m)
