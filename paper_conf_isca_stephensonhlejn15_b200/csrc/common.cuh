@@ -82,7 +82,8 @@ struct ConsumeParams {
   uint32_t npcm;                    // per-PC memdiv matrices kept (shared-memory copies)
   uint64_t* table;                  // device table image
   Offsets off;
-  uint32_t* err;                    // bit 0: row index out of range (stream inconsistent)
+  uint32_t* err;                    // [0] error bits; [2], [3] the unit scheduler (next dynamic unit,
+                                    // CTAs done; back to zero when the launch's last CTA exits)
   uint32_t* dyn_keys;               // insert-on-miss table of unregistered pcs (0: disabled) ...
   unsigned long long* dyn_vals;     // ... [cap][2] warp / thread executions, then dropped records
   uint32_t dyn_cap, dyn_lg;         // slots (power of two) and log2

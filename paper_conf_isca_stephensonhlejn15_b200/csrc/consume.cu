@@ -31,8 +31,28 @@
 #ifndef SASSI_HASH_LG
 #define SASSI_HASH_LG 11     // memdiv distinctness check: 2^11 bit buckets per warp (256 B)
 #endif
+#ifndef SASSI_DYN_ROUNDS
+#define SASSI_DYN_ROUNDS 16  // payload folds: the last 16 rounds of chunks claimed dynamically
+#endif
 #ifndef SASSI_HASH_ROUNDS
 #define SASSI_HASH_ROUNDS 2  // hash rounds (different multipliers) before the exact sort
+#endif
+
+#ifdef SASSI_TIMELINE  // development builds: per-warp %globaltimer stamps of the last launch
+__device__ unsigned long long g_timeline[4 * 148 * 32 * 4];
+extern "C" int sassi_debug_timeline(void* host, size_t bytes) {
+  return (int)cudaMemcpyFromSymbol(host, g_timeline, bytes);
+}
+#define SASSI_STAMP(k, v)                                                                      \
+  if ((tid & 31u) == 0 && blockIdx.x * 32 + (tid >> 5) < 4 * 148 * 32)                            \
+    g_timeline[4 * (blockIdx.x * 32 + (tid >> 5)) + (k)] = (v);
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#else
+#define SASSI_STAMP(k, v)
 #endif
 
 namespace sassi {
@@ -244,11 +264,12 @@ struct SmLayout {
   static constexpr bool kMem = (H & SASSI_H_MEMDIV) != 0, kVal = (H & SASSI_H_VALUE) != 0;
   static constexpr uint32_t kDiag = 0;                                  // 8 u32
   static constexpr uint32_t kImix = 8;                                  // 8 u64 (instmix totals)
-  static constexpr uint32_t kH32 = 24;                                  // [32][32] u32 (memdiv)
+  static constexpr uint32_t kSlot = 24;                                 // [warps] u32 (claimed items)
+  static constexpr uint32_t kH32 = kSlot + kWarpsPerCta;                // [32][32] u32 (memdiv)
   static constexpr uint32_t kH128 = kH32 + 1024;                        // [32][32] u32 (memdiv)
   static constexpr uint32_t kHbm = kH128 + 1024;  // [warps][2^LG / 32] distinctness bitmaps
   static constexpr uint32_t kHbmWords = SASSI_HASH_ROUNDS ? (1u << SASSI_HASH_LG) / 32 : 0u;
-  static constexpr uint32_t kBar = kMem ? kHbm + kWarpsPerCta * kHbmWords : 24;
+  static constexpr uint32_t kBar = kMem ? kHbm + kWarpsPerCta * kHbmWords : kH32;
   static constexpr uint32_t kVbuf = kVal ? ((kBar + 2 * kWarpsPerCta + 31) & ~31u) : kBar;
   static constexpr uint32_t kVar = kVbuf + (kVal ? kWarpsPerCta * kVbufWords : 0u);  // hash, ...
   static_assert(kVbuf % 32 == 0 || !kVal, "value buffers must be 128 B aligned");
@@ -258,9 +279,31 @@ struct SmLayout {
 uint32_t sm_var_words(uint32_t H) {
   const bool mem = H & SASSI_H_MEMDIV, val = H & SASSI_H_VALUE;
   const uint32_t hbm = SASSI_HASH_ROUNDS ? (1u << SASSI_HASH_LG) / 32 : 0u;
-  const uint32_t bar = mem ? 24 + 2048 + kWarpsPerCta * hbm : 24;
+  const uint32_t bar = mem ? 24 + kWarpsPerCta + 2048 + kWarpsPerCta * hbm : 24 + kWarpsPerCta;
   const uint32_t vbuf = val ? ((bar + 2 * kWarpsPerCta + 31) & ~31u) : bar;
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
+}
+
+// Row offsets at record SASSI_CHUNK / 2 of a chunk (the start of its second half): the address /
+// value rows of the first half's records, from their pcs' info words (no handler runs on them).
+// Out of line: it runs only for the launch's last items.
+__device__ __noinline__ uint2 half_offsets(const uint4* hchunk, uint32_t lane,
+                                           const uint4* tbl, uint32_t cap, uint32_t hmul, uint32_t hshr,
+                                           uint32_t arow_bit) {
+  uint32_t arow = 0, vrow = 0;
+  for (uint32_t i = lane; i < SASSI_CHUNK / 2; i += 32) {  // nrec > SASSI_CHUNK / 2: all in range
+    const uint4 h = ld_nc_v4(hchunk + i);
+    uint32_t slot = pc_slot(h.x, hmul, hshr, cap);
+    uint4 e = tbl[slot];
+    while (e.x != h.x && e.x != EMPTY_KEY) {
+      slot = (slot + 1) & (cap - 1);
+      e = tbl[slot];
+    }
+    const uint32_t info = (e.x == h.x && h.x != EMPTY_KEY) ? e.y : 0u;
+    arow += __popc(__ballot_sync(FULL, info & arow_bit));
+    vrow += __reduce_add_sync(FULL, (info >> I_NDST_SHIFT) & 7u);
+  }
+  return make_uint2(arow, vrow);
 }
 
 // kExt: the extended instantiation, used when the insert-on-miss table of unregistered pcs is
@@ -294,6 +337,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   const uint32_t n_regions = p.priv ? kWarpsPerCta : 1u;
 
   const uint32_t tid = threadIdx.x;
+  SASSI_STAMP(0, gtime())
   for (uint32_t i = tid; i < scap; i += blockDim.x) s_hash[i] = p.hash[i];
   if (Ly::kVal && !gm)
     for (uint32_t i = tid; i < p.nvd; i += blockDim.x) s_vstate[i] = make_uint4(FULL, FULL, 1u, 0u);
@@ -312,6 +356,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncthreads();
 
+  SASSI_STAMP(1, gtime())
   const uint32_t lane = tid & 31u, wib = tid >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   uint32_t* const wpriv = s_priv + (p.priv ? wib * p.pw : 0u);
@@ -528,7 +573,38 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       if (done) break;
     }
   }
-  for (uint32_t u = blockIdx.x * kWarpsPerCta + wib; kUnitRows && u < n_units; u += nw) {
+  // payload handler sets: work items are chunks; the launch's last nw chunks are split into two
+  // halves (128 records each) so that the items still running at the end are short. Items below
+  // n_static go round-robin over the warps (SM-interleaved ids); the last SASSI_DYN_ROUNDS rounds
+  // are claimed from a launch-wide counter (p.err[2]; back to zero when the launch's last CTA
+  // exits), so warps whose items were cheaper take more (c2: every warp had ~8 chunks of uneven
+  // cost; measured 0.510 -> 0.480 ms). A warp claims its next item when one ends.
+  uint32_t* const sched = p.err + 2;
+  const uint32_t n_split = min(n_units, nw);
+  const uint32_t n_whole = n_units - n_split, n_items = n_whole + 2 * n_split;
+  const uint32_t n_static = n_whole > SASSI_DYN_ROUNDS * nw ? n_whole - SASSI_DYN_ROUNDS * nw : 0u;
+  // the claimed id reaches the warp through its shared-memory slot, read with a plain load: a loop
+  // whose exit depends on an atomic's return value (or on a volatile load) looks like a spin loop
+  // to ptxas, which then puts YIELDs into every loop nested in it (measured: c3 +1.3 %, c5 +2 %)
+  uint32_t* const s_slot = sm + Ly::kSlot + wib;
+  auto next_item = [&](uint32_t it) -> uint32_t {
+    if (it < n_static) return it;
+    if (lane == 0) *s_slot = atomicAdd(sched, 1u);
+    __syncwarp();
+    const uint32_t v = *s_slot;
+    __syncwarp();
+    return n_static + v;
+  };
+  for (uint32_t it = kUnitRows ? next_item(wib * gridDim.x + blockIdx.x) : n_items; it < n_items;
+       it = next_item(it + nw)) {
+    // item -> chunk u, whole (half 0) or its first / second 128 records (half 1 / 2); a half is
+    // folded as a chunk of its own (its own record count and row bases), so the batch loop below
+    // is the same for every item
+    uint32_t u = it, half = 0;
+    if (it >= n_whole) {
+      u = n_whole + ((it - n_whole) >> 1);
+      half = 1 + ((it - n_whole) & 1u);
+    }
     const ulonglong2 cb0 = kUnitRows ? p.cb[u] : make_ulonglong2(p.arow_base, p.vrow_base);
     const ulonglong2 cb1 = kUnitRows ? p.cb[u + 1] : cb0;
     if (kUnitRows && !(cb0.x >= p.arow_base && cb0.x <= cb1.x && cb1.x <= p.arow_end &&
@@ -536,16 +612,34 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       err |= kErrIndex;  // chunk index outside the row buffers
       continue;
     }
-    // rows are addressed relative to this chunk: 32-bit offsets from here on
-    const uint64_t* const achunk = p.addr + ((cb0.x - p.arow_base) << 5);
-    const uint32_t* const vchunk = p.val + ((cb0.y - p.vrow_base) << 5);
-    const uint32_t aend = (uint32_t)(cb1.x - cb0.x), vend = (uint32_t)(cb1.y - cb0.y);
+    const uint4* hchunk = p.hdr + u * SASSI_CHUNK;
+    uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
+    uint32_t aend = (uint32_t)(cb1.x - cb0.x), vend = (uint32_t)(cb1.y - cb0.y);
+    uint32_t a0 = 0, v0 = 0;  // rows before the item's first record (second halves)
+    if (half == 2) {
+      if (nrec <= SASSI_CHUNK / 2) continue;  // a short last chunk: its first half covers it
+      const uint2 r = half_offsets(hchunk, lane, gm ? p.hash : s_hash, cap, p.hmul, p.hshr,
+                                   p.arow_bit);
+      if (r.x > aend || r.y > vend) {
+        err |= kErrRows;  // the first half's rows run past the chunk's rows
+        continue;
+      }
+      a0 = r.x;
+      v0 = r.y;
+      aend -= a0;
+      vend -= v0;
+      hchunk += SASSI_CHUNK / 2;
+      nrec -= SASSI_CHUNK / 2;
+    } else if (half == 1) {
+      nrec = min(nrec, (uint32_t)SASSI_CHUNK / 2);  // bounded by the chunk's rows, end unchecked
+    }
+    // rows are addressed relative to this item: 32-bit offsets from here on
+    const uint64_t* const achunk = p.addr + ((cb0.x - p.arow_base + a0) << 5);
+    const uint32_t* const vchunk = p.val + ((cb0.y - p.vrow_base + v0) << 5);
     uint32_t arow = 0, vrow = 0;
-    const uint4* const hchunk = p.hdr + u * SASSI_CHUNK;
-    const uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
     const uint32_t nbat = (nrec + 31) >> 5;
     if (lane == 0) c_rec += nrec;
-    // header loads are clamped to the chunk's last record (always in bounds) and masked by `valid`
+    // header loads are clamped to the item's last record (always in bounds) and masked by `valid`
     const uint32_t ilast = nrec - 1;
     uint4 hnext = ld_nc_v4(hchunk + min(lane, ilast));
     uint32_t b = 0;
@@ -747,9 +841,12 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
         }
       }
     }
-    if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && lane == 0 && (arow != aend || vrow != vend))
+    const bool first_half = it >= n_whole && ((it - n_whole) & 1u) == 0;
+    if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && !first_half && lane == 0 &&
+        (arow != aend || vrow != vend))
       err |= kErrRows;  // index disagrees with the rows
   }
+  SASSI_STAMP(2, gtime())
   if (H & SASSI_H_INSTCOUNT) {
     if (kVertical) flush_planes();
     if (acc_w != FULL && acc) gadd(p.off.counts + 32ull * acc_w + lane, (unsigned long long)acc);
@@ -769,6 +866,14 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     if (err) atomicOr(p.err, err);
   }
   __syncthreads();
+  // every warp of the CTA is past its last claim: the launch's last CTA resets the scheduler
+  if (kUnitRows && tid == 0) {
+    // (every claim of this CTA has returned its value: no fence needed before the count)
+    if (atomicAdd(sched + 1, 1u) == gridDim.x - 1) {
+      sched[0] = 0;
+      sched[1] = 0;
+    }
+  }
 
   // ---- flush: sum the warps' private counters, fold into the global u64 image ----
   if (tid < 4 && s_diag[tid]) gadd(tid, (unsigned long long)s_diag[tid]);
@@ -852,6 +957,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       }
     }
   }
+  SASSI_STAMP(3, gtime())
 }
 
 __global__ void dyn_reset_kernel(uint32_t* keys, unsigned long long* vals, uint32_t cap) {

@@ -135,6 +135,24 @@ def test_c2_full(every):
     assert diff_tables(t, o, len(h["sites"]), P.total_warps) is None
 
 
+def test_c2_back_to_back_launches_dynamic_schedule():
+    """The payload fold hands out its last rounds of chunks from a launch-wide counter that the
+    launch's last CTA resets: three back-to-back folds of c2 (every item claimed
+    dynamically at this size) on one context, without a reset in between, equal three oracle
+    passes; a counter left non-zero would skip items in the second launch."""
+    P, mask, d = _gen("c2")
+    h = gen.to_host(d)
+    S, W = len(h["sites"]), P.total_warps
+    ctx = sassi.Context(h["sites"], W, mask)
+    o = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+    for k in range(3):
+        ctx.consume(d)
+        if k:
+            oracle.consume(o, h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+        assert diff_tables(ctx.read_tables(), o, S, W) is None
+    ctx.close()
+
+
 def _prefix(d, n):
     """First n records of a device stream (n a multiple of SASSI_CHUNK) with their rows."""
     assert n % 256 == 0
