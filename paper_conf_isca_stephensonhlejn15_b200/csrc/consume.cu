@@ -31,6 +31,9 @@
 #ifndef SASSI_HASH_LG
 #define SASSI_HASH_LG 11     // memdiv distinctness check: 2^11 bit buckets per warp (256 B)
 #endif
+#ifndef SASSI_SPLIT_PARTS
+#define SASSI_SPLIT_PARTS 2  // the launch's last chunks are folded in this many parts
+#endif
 #ifndef SASSI_DYN_ROUNDS
 #define SASSI_DYN_ROUNDS 16  // payload folds: the last 16 rounds of chunks claimed dynamically
 #endif
@@ -284,14 +287,14 @@ uint32_t sm_var_words(uint32_t H) {
   return vbuf + (val ? kWarpsPerCta * kVbufWords : 0u);
 }
 
-// Row offsets at record SASSI_CHUNK / 2 of a chunk (the start of its second half): the address /
-// value rows of the first half's records, from their pcs' info words (no handler runs on them).
-// Out of line: it runs only for the launch's last items.
-__device__ __noinline__ uint2 half_offsets(const uint4* hchunk, uint32_t lane,
+// Row offsets at record r0 of a chunk (the start of one of its parts, r0 a multiple of 32 below
+// the chunk's record count): the address / value rows of records [0, r0), from their pcs' info
+// words (no handler runs on them). Out of line: it runs only for the launch's last items.
+__device__ __noinline__ uint2 part_offsets(const uint4* hchunk, uint32_t r0, uint32_t lane,
                                            const uint4* tbl, uint32_t cap, uint32_t hmul, uint32_t hshr,
                                            uint32_t arow_bit) {
   uint32_t arow = 0, vrow = 0;
-  for (uint32_t i = lane; i < SASSI_CHUNK / 2; i += 32) {  // nrec > SASSI_CHUNK / 2: all in range
+  for (uint32_t i = lane; i < r0; i += 32) {
     const uint4 h = ld_nc_v4(hchunk + i);
     uint32_t slot = pc_slot(h.x, hmul, hshr, cap);
     uint4 e = tbl[slot];
@@ -581,7 +584,8 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   // cost; measured 0.510 -> 0.480 ms). A warp claims its next item when one ends.
   uint32_t* const sched = p.err + 2;
   const uint32_t n_split = min(n_units, nw);
-  const uint32_t n_whole = n_units - n_split, n_items = n_whole + 2 * n_split;
+  constexpr uint32_t kParts = SASSI_SPLIT_PARTS, kPartRec = SASSI_CHUNK / kParts;
+  const uint32_t n_whole = n_units - n_split, n_items = n_whole + kParts * n_split;
   const uint32_t n_static = n_whole > SASSI_DYN_ROUNDS * nw ? n_whole - SASSI_DYN_ROUNDS * nw : 0u;
   // the claimed id reaches the warp through its shared-memory slot, read with a plain load: a loop
   // whose exit depends on an atomic's return value (or on a volatile load) looks like a spin loop
@@ -597,13 +601,13 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   };
   for (uint32_t it = kUnitRows ? next_item(wib * gridDim.x + blockIdx.x) : n_items; it < n_items;
        it = next_item(it + nw)) {
-    // item -> chunk u, whole (half 0) or its first / second 128 records (half 1 / 2); a half is
-    // folded as a chunk of its own (its own record count and row bases), so the batch loop below
-    // is the same for every item
-    uint32_t u = it, half = 0;
+    // item -> chunk u, whole or one of its kParts parts (records [part * kPartRec, + kPartRec));
+    // a part is folded as a chunk of its own (its own record count and row bases), so the batch
+    // loop below is the same for every item
+    uint32_t u = it, part = 0;
     if (it >= n_whole) {
-      u = n_whole + ((it - n_whole) >> 1);
-      half = 1 + ((it - n_whole) & 1u);
+      u = n_whole + (it - n_whole) / kParts;
+      part = (it - n_whole) % kParts;
     }
     const ulonglong2 cb0 = kUnitRows ? p.cb[u] : make_ulonglong2(p.arow_base, p.vrow_base);
     const ulonglong2 cb1 = kUnitRows ? p.cb[u + 1] : cb0;
@@ -615,23 +619,24 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
     const uint4* hchunk = p.hdr + u * SASSI_CHUNK;
     uint32_t nrec = min(p.n - u * SASSI_CHUNK, (uint32_t)SASSI_CHUNK);
     uint32_t aend = (uint32_t)(cb1.x - cb0.x), vend = (uint32_t)(cb1.y - cb0.y);
-    uint32_t a0 = 0, v0 = 0;  // rows before the item's first record (second halves)
-    if (half == 2) {
-      if (nrec <= SASSI_CHUNK / 2) continue;  // a short last chunk: its first half covers it
-      const uint2 r = half_offsets(hchunk, lane, gm ? p.hash : s_hash, cap, p.hmul, p.hshr,
-                                   p.arow_bit);
-      if (r.x > aend || r.y > vend) {
-        err |= kErrRows;  // the first half's rows run past the chunk's rows
-        continue;
+    uint32_t a0 = 0, v0 = 0;  // rows before the item's first record (parts after the first)
+    if (it >= n_whole) {
+      const uint32_t r0 = part * kPartRec;
+      if (nrec <= r0) continue;  // a short last chunk: its earlier parts cover it
+      if (r0) {
+        const uint2 r = part_offsets(hchunk, r0, lane, gm ? p.hash : s_hash, cap, p.hmul, p.hshr,
+                                     p.arow_bit);
+        if (r.x > aend || r.y > vend) {
+          err |= kErrRows;  // the earlier parts' rows run past the chunk's rows
+          continue;
+        }
+        a0 = r.x;
+        v0 = r.y;
+        aend -= a0;
+        vend -= v0;
+        hchunk += r0;
       }
-      a0 = r.x;
-      v0 = r.y;
-      aend -= a0;
-      vend -= v0;
-      hchunk += SASSI_CHUNK / 2;
-      nrec -= SASSI_CHUNK / 2;
-    } else if (half == 1) {
-      nrec = min(nrec, (uint32_t)SASSI_CHUNK / 2);  // bounded by the chunk's rows, end unchecked
+      nrec = min(nrec - r0, kPartRec);  // bounded by the chunk's rows; the end checked by the last part
     }
     // rows are addressed relative to this item: 32-bit offsets from here on
     const uint64_t* const achunk = p.addr + ((cb0.x - p.arow_base + a0) << 5);
@@ -841,8 +846,11 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
         }
       }
     }
-    const bool first_half = it >= n_whole && ((it - n_whole) & 1u) == 0;
-    if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && !first_half && lane == 0 &&
+    // a part ending before its chunk's last record has no end of its own to check
+    const bool inner_part = it >= n_whole && ((it - n_whole) % kParts + 1) * kPartRec <
+                                                 min(p.n - (n_whole + (it - n_whole) / kParts) * SASSI_CHUNK,
+                                                     (uint32_t)SASSI_CHUNK);
+    if ((H & (SASSI_H_MEMDIV | SASSI_H_VALUE)) && b == nbat && !inner_part && lane == 0 &&
         (arow != aend || vrow != vend))
       err |= kErrRows;  // index disagrees with the rows
   }
