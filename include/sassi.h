@@ -262,7 +262,9 @@ int sassi_read_dynamic_pcs(struct sassi_ctx* ctx, sassi_dyn_pc* host_out, uint32
 
 /* Fold n records (DEVICE buffers) into the context's tables (and, with peer tables attached,
  * into theirs); asynchronous, stream-ordered. Tables accumulate across calls until sassi_reset.
- * One kernel launch per 2^29 records (the
+ * Folds of one context may also run on unordered streams (the table updates are atomic; each
+ * launch has its own chunk-scheduler words, up to 64 launches in flight). One kernel launch per
+ * 2^29 records (the
  * environment variable SASSI_MAX_LAUNCH_RECORDS, read at sassi_ctx_create, lowers that to a
  * multiple of SASSI_CHUNK for tests). Errors: EINVAL, ESTATE (no handler), ECUDA. */
 int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, void* stream);

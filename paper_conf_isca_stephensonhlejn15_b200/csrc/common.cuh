@@ -32,6 +32,10 @@ constexpr uint32_t kMaxPeers = 7;   // fused merge over peer memory: up to 8 GPU
 // chunk's rows or the index disagrees with the rows, 8 = chunk index outside the row buffers
 // (both SASSI_EFORMAT); kMergeMismatch = a merge found other site tables (SASSI_EMISMATCH)
 constexpr uint32_t kErrRows = 4u, kErrIndex = 8u, kMergeMismatch = 1u << 16;
+// the context's error word, then kSchedSlots chunk schedulers of 2 words; consecutive fold launches
+// take consecutive slots, so folds of one context on unordered streams (up to kSchedSlots in
+// flight) never share one
+constexpr uint32_t kSchedSlots = 64, kErrWords = 4 + 2 * kSchedSlots;
 
 // Packed per-site info word in the hash (bit layout). The companion cidx word holds the
 // site's compact branch-or-memdiv slot (low 16 bits) and compact value-site slot (high 16 bits).
@@ -82,8 +86,9 @@ struct ConsumeParams {
   uint32_t npcm;                    // per-PC memdiv matrices kept (shared-memory copies)
   uint64_t* table;                  // device table image
   Offsets off;
-  uint32_t* err;                    // [0] error bits; [2], [3] the unit scheduler (next dynamic unit,
-                                    // CTAs done; back to zero when the launch's last CTA exits)
+  uint32_t* err;                    // error bits (bit 0: row index out of range ...)
+  uint32_t* sched;                  // this launch's chunk scheduler {next claimed item, CTAs done}:
+                                    // zero at launch, back to zero when the launch's last CTA exits
   uint32_t* dyn_keys;               // insert-on-miss table of unregistered pcs (0: disabled) ...
   unsigned long long* dyn_vals;     // ... [cap][2] warp / thread executions, then dropped records
   uint32_t dyn_cap, dyn_lg;         // slots (power of two) and log2
@@ -151,7 +156,8 @@ struct sassi_ctx {
   uint32_t npcm = 0;
   uint64_t site_checksum = 0;       // of the registered sites (checksum adds the selection)
   uint32_t* d_flush = nullptr;      // flush_b | flush_m | flush_v
-  uint32_t* d_err = nullptr;
+  uint32_t* d_err = nullptr;          // [kErrWords]: error bits, chunk schedulers
+  uint64_t sched_seq = 0;             // fold launches so far (scheduler slot rotation)
   uint64_t* d_scan = nullptr;       // sampling: prefix [32W+1] + block sums
   uint64_t scan_words = 0;
   void* d_sample = nullptr;         // sampling: draws + status word of the host-output form

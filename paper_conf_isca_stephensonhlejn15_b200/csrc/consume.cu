@@ -579,10 +579,10 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   // payload handler sets: work items are chunks; the launch's last nw chunks are split into two
   // halves (128 records each) so that the items still running at the end are short. Items below
   // n_static go round-robin over the warps (SM-interleaved ids); the last SASSI_DYN_ROUNDS rounds
-  // are claimed from a launch-wide counter (p.err[2]; back to zero when the launch's last CTA
+  // are claimed from a launch-wide counter (p.sched[0]; back to zero when the launch's last CTA
   // exits), so warps whose items were cheaper take more (c2: every warp had ~8 chunks of uneven
   // cost; measured 0.510 -> 0.480 ms). A warp claims its next item when one ends.
-  uint32_t* const sched = p.err + 2;
+  uint32_t* const sched = p.sched;
   const uint32_t n_split = min(n_units, nw);
   constexpr uint32_t kParts = SASSI_SPLIT_PARTS, kPartRec = SASSI_CHUNK / kParts;
   const uint32_t n_whole = n_units - n_split, n_items = n_whole + kParts * n_split;
@@ -1055,7 +1055,9 @@ int launch_consume(sassi_ctx* c, const ConsumeParams& p, cudaStream_t s) {
   uint64_t grid = (uint64_t)c->num_sms * per_sm;
   const uint64_t need = (units + kWarpsPerCta - 1) / kWarpsPerCta;
   if (grid > need) grid = need ? need : 1;
-  fn<<<(unsigned)grid, kConsumeThreads, c->smem_bytes, s>>>(p);
+  ConsumeParams q = p;
+  q.sched = c->d_err + 4 + 2 * (c->sched_seq++ % kSchedSlots);
+  fn<<<(unsigned)grid, kConsumeThreads, c->smem_bytes, s>>>(q);
   SASSI_CUDA(cudaGetLastError());
   c->launches += 1;
   return SASSI_OK;

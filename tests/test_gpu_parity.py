@@ -153,6 +153,27 @@ def test_c2_back_to_back_launches_dynamic_schedule():
     ctx.close()
 
 
+def test_concurrent_folds_on_two_streams():
+    """Two folds of c2 into one context on two unordered streams (each launch has its own
+    chunk-scheduler words): the tables equal two oracle passes."""
+    import torch
+    P, mask, d = _gen("c2", limit=3_000_000)
+    h = gen.to_host(d)
+    S, W = len(h["sites"]), P.total_warps
+    ctx = sassi.Context(h["sites"], W, mask)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    for _ in range(3):
+        ctx.consume(d, stream=s1)
+        ctx.consume(d, stream=s2)
+    torch.cuda.synchronize()
+    o = oracle.run(h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+    for _ in range(5):
+        oracle.consume(o, h["sites"], W, mask, h["hdr"], h["addr"], h["val"])
+    assert diff_tables(ctx.read_tables(), o, S, W) is None
+    ctx.close()
+
+
 def _prefix(d, n):
     """First n records of a device stream (n a multiple of SASSI_CHUNK) with their rows."""
     assert n % 256 == 0
