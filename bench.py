@@ -828,7 +828,9 @@ def measure_e2e(rec, P, mask, n_e2e, dev, comm=None, world=1, launched=False, gl
     if cm is not None:
         sassi.sassi_nccl_comm_destroy(cm)
     ctx.close()
-    h2d = 16 * n_e2e + 256 * na + 128 * nv + 16 * (n_e2e // 256 + 1)
+    # what sassi_consume_host copies: rows only for the handlers that read them (sassi.h)
+    h2d = (16 * n_e2e + (256 * na if mask & 2 else 0) + (128 * nv if mask & 4 else 0) +
+           (16 * (n_e2e // 256 + 1) if mask & 6 else 0))
     return {"value": world * reps * n_e2e / el, "unit": "records/s", "h2d_bytes_per_step": world * h2d,
             "d2h_bytes_per_step": world * 8 * ctx.layout["total"], "records_per_step": world * n_e2e,
             "h2d_gbs": world * reps * h2d / el / 1e9,

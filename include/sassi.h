@@ -271,7 +271,9 @@ int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, 
 
 /* Same fold from HOST buffers (pinned or pageable): the library copies slices to the device
  * (double-buffered on `stream` plus an internal copy stream), consumes them, and returns after
- * the stream work completes. recs->chunk_base is required (host). */
+ * the stream work completes. recs->chunk_base is required (host). Only what the attached handlers
+ * read crosses PCIe: address rows with SASSI_H_MEMDIV, value rows with SASSI_H_VALUE, the chunk
+ * index with either; header-only handler sets copy the headers alone. */
 int sassi_consume_host(struct sassi_ctx* ctx, const sassi_records* host_recs, uint64_t n,
                        void* stream);
 

@@ -370,14 +370,35 @@ def test_reset_and_accumulate():
     ctx.close()
 
 
-def test_consume_host_equals_device():
-    P, mask, d = _gen("c2", limit=3_000_000)
+@pytest.mark.parametrize("mask", [15, 1, 2, 4, 6, 8, 31])
+def test_consume_host_equals_device(mask):
+    """sassi_consume_host copies only what the attached handlers read (address rows for memdiv,
+    value rows for value, the chunk index for either): every handler set folds from host buffers
+    to the device fold's tables."""
+    P, _, d = _gen("c2", limit=3_000_000)
     h = gen.to_host(d)
     t_dev = gpu_table(h["sites"], P.total_warps, mask, d)
     ctx = sassi.Context(h["sites"], P.total_warps, mask)
     hrec = dict(hdr=np.ascontiguousarray(h["hdr"]), addr=h["addr"], val=h["val"],
                 chunk_base=h["chunk_base"], n=h["n"], n_addr_rows=h["n_addr_rows"],
                 n_val_rows=h["n_val_rows"])
+    ctx.consume_host(hrec)
+    assert np.array_equal(ctx.read_tables(), t_dev)
+    ctx.close()
+
+
+def test_consume_host_header_only_reads_no_rows():
+    """A header-only handler set (per-thread counts, the injection-profiling pass) folds from the
+    headers alone: the host row buffers passed here hold one row each while the record counts
+    say millions, so any copy of rows would read far past them."""
+    P, _, d = _gen("c2", limit=3_000_000)
+    h = gen.to_host(d)
+    mask = sassi.SASSI_H_INSTCOUNT
+    t_dev = gpu_table(h["sites"], P.total_warps, mask, d)
+    ctx = sassi.Context(h["sites"], P.total_warps, mask)
+    hrec = dict(hdr=np.ascontiguousarray(h["hdr"]), addr=np.zeros((1, 32), np.uint64),
+                val=np.zeros((1, 32), np.uint32), chunk_base=h["chunk_base"], n=h["n"],
+                n_addr_rows=h["n_addr_rows"], n_val_rows=h["n_val_rows"])
     ctx.consume_host(hrec)
     assert np.array_equal(ctx.read_tables(), t_dev)
     ctx.close()
