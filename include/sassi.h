@@ -266,7 +266,9 @@ int sassi_read_dynamic_pcs(struct sassi_ctx* ctx, sassi_dyn_pc* host_out, uint32
  * launch has its own chunk-scheduler words, up to 64 launches in flight). One kernel launch per
  * 2^29 records (the
  * environment variable SASSI_MAX_LAUNCH_RECORDS, read at sassi_ctx_create, lowers that to a
- * multiple of SASSI_CHUNK for tests). Errors: EINVAL, ESTATE (no handler), ECUDA. */
+ * multiple of SASSI_CHUNK for tests). hdr, addr, val and chunk_base must be 16-byte aligned
+ * (vector loads, TMA bulk copies and bulk L2 prefetches read them). Errors: EINVAL (incl.
+ * misaligned buffers), ESTATE (no handler), ECUDA. */
 int sassi_consume(struct sassi_ctx* ctx, const sassi_records* recs, uint64_t n, void* stream);
 
 /* Same fold from HOST buffers (pinned or pageable): the library copies slices to the device

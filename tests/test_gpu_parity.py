@@ -71,6 +71,28 @@ def test_empty_stream():
     assert np.array_equal(t, oracle.table_init(len(s), T0.N_WARPS, oracle.H_ALL))
 
 
+def test_misaligned_buffers_are_rejected():
+    """Headers are vector-loaded, value rows TMA-copied and address rows bulk-prefetched: every
+    buffer must be 16-byte aligned, and an 8-byte offset one is refused with EINVAL up front."""
+    import torch
+    s = T0.sites()
+    hdr, addr, val = T0.records()
+    d = to_device(s, hdr, addr, val)
+    ctx = sassi.Context(s, T0.N_WARPS, sassi.SASSI_H_ALL)
+    for key in ("hdr", "addr", "val", "chunk_base"):
+        t = d[key]
+        buf = torch.empty(t.numel() * t.element_size() + 8, dtype=torch.uint8, device=t.device)
+        moved = buf[8:].view(t.dtype).reshape(t.shape)
+        moved.copy_(t)
+        with pytest.raises(sassi.SassiError) as ei:
+            ctx.consume(dict(d, **{key: moved}))
+        assert ei.value.status == sassi.SASSI_EINVAL and "aligned" in str(ei.value)
+    ctx.consume(d)  # the aligned originals still fold
+    assert np.array_equal(ctx.read_tables(),
+                          oracle.run(s, T0.N_WARPS, oracle.H_ALL, hdr, addr, val))
+    ctx.close()
+
+
 def test_inconsistent_chunk_index_is_reported():
     s, W, hdr, addr, val = random_trace(77, n=3000)
     cb = host_chunk_base(s, hdr)
