@@ -579,8 +579,9 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
       if (done) break;
     }
   }
-  // payload handler sets: work items are chunks; the launch's last nw chunks are split into two
-  // halves (128 records each) so that the items still running at the end are short. Items below
+  // payload handler sets: work items are chunks; the launch's last nw chunks are split into
+  // SASSI_SPLIT_PARTS parts (128 records each) so that the items still running at the end are
+  // short. Items below
   // n_static go round-robin over the warps (SM-interleaved ids); the last SASSI_DYN_ROUNDS rounds
   // are claimed from a launch-wide counter (p.sched[0]; back to zero when the launch's last CTA
   // exits), so warps whose items were cheaper take more (c2: every warp had ~8 chunks of uneven
@@ -588,6 +589,7 @@ __global__ void __launch_bounds__(kConsumeThreads, 1) consume_kernel(const Consu
   uint32_t* const sched = p.sched;
   const uint32_t n_split = min(n_units, nw);
   constexpr uint32_t kParts = SASSI_SPLIT_PARTS, kPartRec = SASSI_CHUNK / kParts;
+  static_assert(kPartRec % 32 == 0 && kPartRec * kParts == SASSI_CHUNK, "parts of whole batches");
   const uint32_t n_whole = n_units - n_split, n_items = n_whole + kParts * n_split;
   const uint32_t n_static = n_whole > SASSI_DYN_ROUNDS * nw ? n_whole - SASSI_DYN_ROUNDS * nw : 0u;
   // the claimed id reaches the warp through its shared-memory slot, read with a plain load: a loop
