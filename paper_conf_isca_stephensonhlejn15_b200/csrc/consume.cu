@@ -29,7 +29,7 @@
 #define SASSI_ROW_GROUP 3  // memdiv address rows loaded per group (measured: 3 beats 2, 4, 6)
 #endif
 #ifndef SASSI_HASH_LG
-#define SASSI_HASH_LG 11     // memdiv distinctness check: 2^11 bit buckets per warp (256 B)
+#define SASSI_HASH_LG 12     // memdiv distinctness check: 2^12 bit buckets per warp (512 B)
 #endif
 #ifndef SASSI_PREF_ROWS
 #define SASSI_PREF_ROWS 6  // memdiv: address rows of the next batch prefetched into L2 (0: off)
